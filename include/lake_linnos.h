@@ -186,6 +186,14 @@ int lake_linnos_infer_host(const void *h_in, uint32_t flags, int64_t n, int32_t 
 uint64_t lake_linnos_launch_count(void);
 void lake_linnos_reset_launch_count(void);
 
+/* Device-side timing of the fused MLP kernel (the dominant kernel), for the bench's
+ * roofline: while enabled, every fused-kernel launch by _infer / _multi_grouped is
+ * bracketed by two CUDA events recorded on the launch stream. _profile_read waits for
+ * the recorded events, returns the summed elapsed milliseconds and the number of
+ * bracketed launches, and resets the accumulator. Enabling also resets it. */
+int lake_linnos_profile_enable(int enable);
+int lake_linnos_profile_read(double *total_ms, int64_t *n_launches);
+
 /* Static string for a status code; never NULL. */
 const char *lake_linnos_strerror(int status);
 

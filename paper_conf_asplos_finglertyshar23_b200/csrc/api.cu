@@ -1,0 +1,603 @@
+// api.cu — the C ABI (include/lake_linnos.h): argument validation, per-device model
+// registry, weight-image preparation, dispatch to the kernels. See the header for the
+// contract of every function; PAPER.md citations are there.
+//
+// Model registry: one DevModel table of LAKE_MAX_MODELS slots per CUDA device, mirrored
+// on the host (for validation without a device round trip) and in device memory (for the
+// multi-model kernels, which look a tile's model up by slot). A slot is the model_id — one
+// model per block device, as the paper's per-device registries.
+#include <cuda_bf16.h>
+#include <cuda_fp16.h>
+
+#include <atomic>
+#include <cmath>
+#include <cstring>
+#include <mutex>
+#include <new>
+#include <vector>
+
+#include "lake_internal.h"
+
+namespace lake {
+
+static std::atomic<uint64_t> g_launches{0};
+void count_launch(int k) { g_launches.fetch_add((uint64_t)k, std::memory_order_relaxed); }
+
+namespace {
+
+constexpr int kMaxDevices = 64;
+
+struct ModelBufs {
+  void *fp32 = nullptr;
+  void *tc = nullptr;
+};
+
+struct DeviceState {
+  bool init = false;
+  DevModel host[LAKE_MAX_MODELS];
+  ModelBufs bufs[LAKE_MAX_MODELS];
+  DevModel *table = nullptr;  // device copy
+};
+
+std::mutex g_mu;
+DeviceState *g_dev[kMaxDevices] = {nullptr};
+
+// profiling of the main MLP kernel launches (bench roofline)
+std::mutex g_prof_mu;
+bool g_prof = false;
+std::vector<std::pair<cudaEvent_t, cudaEvent_t>> g_prof_ev;
+size_t g_prof_used = 0;
+
+int nh_of(int32_t arch) { return arch + 1; }
+
+size_t blob_floats(int32_t arch) {
+  switch (arch) {
+    case LAKE_ARCH_NN: return 256 * 31 + 256 + 2 * 256 + 2;
+    case LAKE_ARCH_NN1: return 256 * 31 + 256 + 256 * 256 + 256 + 2 * 256 + 2;
+    case LAKE_ARCH_NN2: return 256 * 31 + 256 + 2 * (256 * 256 + 256) + 2 * 256 + 2;
+    default: return 0;
+  }
+}
+
+// Returns the state for `device`, creating the device table on first use.
+// Caller holds g_mu and has made `device` current.
+int get_state(int device, DeviceState **out) {
+  if (device < 0 || device >= kMaxDevices) return LAKE_ERR_INVAL;
+  DeviceState *st = g_dev[device];
+  if (!st) {
+    st = new (std::nothrow) DeviceState();
+    if (!st) return LAKE_ERR_NOMEM;
+    for (int i = 0; i < LAKE_MAX_MODELS; ++i) {
+      std::memset(&st->host[i], 0, sizeof(DevModel));
+      st->host[i].arch = -1;
+    }
+    g_dev[device] = st;
+  }
+  if (!st->init) {
+    if (cudaMalloc(&st->table, sizeof(DevModel) * LAKE_MAX_MODELS) != cudaSuccess)
+      return LAKE_ERR_NOMEM;
+    if (cudaMemcpy(st->table, st->host, sizeof(DevModel) * LAKE_MAX_MODELS,
+                   cudaMemcpyHostToDevice) != cudaSuccess)
+      return LAKE_ERR_CUDA;
+    st->init = true;
+  }
+  *out = st;
+  return LAKE_OK;
+}
+
+// Permuted column position for the FP32 path (see lake_internal.h).
+inline int perm_col(int j) {
+  const int tc = j & 31, jj = j >> 5;
+  return (jj >> 2) * 128 + tc * 4 + (jj & 3);
+}
+
+struct BlobView {
+  const float *W[4];
+  const float *b[4];
+  int nh;
+};
+
+BlobView view_blob(int32_t arch, const float *blob) {
+  BlobView v{};
+  v.nh = nh_of(arch);
+  const float *p = blob;
+  v.W[0] = p; p += 256 * 31;
+  v.b[0] = p; p += 256;
+  for (int l = 1; l < v.nh; ++l) {
+    v.W[l] = p; p += 256 * 256;
+    v.b[l] = p; p += 256;
+  }
+  v.W[v.nh] = p; p += 2 * 256;
+  v.b[v.nh] = p;
+  return v;
+}
+
+// UMMA K-major SWIZZLE_NONE offset (bytes) of element (row r, k) in an R-row operand.
+inline size_t umma_off(int r, int k, int R) {
+  return (size_t)(k >> 3) * (R * 16) + (size_t)r * 16 + (size_t)(k & 7) * 2;
+}
+
+template <typename T>
+inline uint16_t to_bits(float v);
+template <>
+inline uint16_t to_bits<__half>(float v) {
+  __half h = __float2half_rn(v);
+  uint16_t u;
+  std::memcpy(&u, &h, 2);
+  return u;
+}
+template <>
+inline uint16_t to_bits<__nv_bfloat16>(float v) {
+  __nv_bfloat16 h = __float2bfloat16_rn(v);
+  uint16_t u;
+  std::memcpy(&u, &h, 2);
+  return u;
+}
+
+template <typename T>
+void build_tc_image(const BlobView &v, uint8_t *img /* 2 * bytes */, size_t bytes) {
+  std::memset(img, 0, 2 * bytes);
+  const int nh = v.nh;
+  for (int rank = 0; rank < 2; ++rank) {
+    uint8_t *base = img + rank * bytes;
+    auto put = [&](size_t off, float val) {
+      const uint16_t u = to_bits<T>(val);
+      std::memcpy(base + off, &u, 2);
+    };
+    for (int n = 0; n < 128; ++n)
+      for (int k = 0; k < kTcK0; ++k)
+        put(umma_off(n, k, 128), k < 31 ? v.W[0][(size_t)(rank * 128 + n) * 31 + k] : 0.0f);
+    for (int l = 1; l < nh; ++l) {
+      const size_t o = kTcW0HalfBytes + (size_t)(l - 1) * kTcWhHalfBytes;
+      for (int n = 0; n < 128; ++n)
+        for (int k = 0; k < 256; ++k)
+          put(o + umma_off(n, k, 128), v.W[l][(size_t)(rank * 128 + n) * 256 + k]);
+    }
+    const size_t wo = kTcW0HalfBytes + (size_t)(nh - 1) * kTcWhHalfBytes;
+    for (int n = 0; n < kTcOutN / 2; ++n) {
+      const int o = rank * (kTcOutN / 2) + n;
+      for (int k = 0; k < 256; ++k) put(wo + umma_off(n, k, kTcOutN / 2), o < 2 ? v.W[nh][o * 256 + k] : 0.0f);
+    }
+    float *bias = reinterpret_cast<float *>(base + wo + kTcWoHalfBytes);
+    for (int l = 0; l < nh; ++l) std::memcpy(bias + l * 256, v.b[l], 256 * 4);
+    bias[nh * 256 + 0] = v.b[nh][0];
+    bias[nh * 256 + 1] = v.b[nh][1];
+  }
+}
+
+void free_bufs(ModelBufs &b) {
+  if (b.fp32) cudaFree(b.fp32);
+  if (b.tc) cudaFree(b.tc);
+  b.fp32 = b.tc = nullptr;
+}
+
+int cuda_status(cudaError_t e) {
+  if (e == cudaSuccess) return LAKE_OK;
+  if (e == cudaErrorMemoryAllocation) return LAKE_ERR_NOMEM;
+  return LAKE_ERR_CUDA;
+}
+
+struct DeviceGuard {
+  int prev = -1;
+  bool ok = true;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) { ok = false; return; }
+    if (prev != dev && cudaSetDevice(dev) != cudaSuccess) ok = false;
+  }
+  ~DeviceGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+
+// Look up a loaded model on the current device (validation for infer*).
+int current_model(int32_t model_id, int *device, DevModel *out, const DevModel **table) {
+  if (model_id < 0 || model_id >= LAKE_MAX_MODELS) return LAKE_ERR_NOMODEL;
+  if (cudaGetDevice(device) != cudaSuccess) return LAKE_ERR_CUDA;
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (*device < 0 || *device >= kMaxDevices || !g_dev[*device] || !g_dev[*device]->init)
+    return LAKE_ERR_NOMODEL;
+  const DevModel &m = g_dev[*device]->host[model_id];
+  if (m.arch < 0) return LAKE_ERR_NOMODEL;
+  *out = m;
+  if (table) *table = g_dev[*device]->table;
+  return LAKE_OK;
+}
+
+int current_table(int *device, const DevModel **table, int *any) {
+  if (cudaGetDevice(device) != cudaSuccess) return LAKE_ERR_CUDA;
+  std::lock_guard<std::mutex> lk(g_mu);
+  *any = 0;
+  if (*device < 0 || *device >= kMaxDevices || !g_dev[*device] || !g_dev[*device]->init) {
+    *table = nullptr;
+    return LAKE_OK;
+  }
+  *table = g_dev[*device]->table;
+  for (int i = 0; i < LAKE_MAX_MODELS; ++i)
+    if (g_dev[*device]->host[i].arch >= 0) { *any = 1; break; }
+  return LAKE_OK;
+}
+
+int check_flags(uint32_t flags, int64_t n, int *in_kind, int *prec) {
+  if (flags & ~(uint32_t)(LAKE_IN_MASK | LAKE_PREC_MASK)) return LAKE_ERR_INVAL;
+  *in_kind = (int)(flags & LAKE_IN_MASK);
+  const uint32_t p = flags & LAKE_PREC_MASK;
+  switch (p) {
+    case LAKE_PREC_FP32: *prec = -1; break;
+    case LAKE_PREC_F16: *prec = 0; break;
+    case LAKE_PREC_BF16: *prec = 1; break;
+    case LAKE_PREC_TF32: return LAKE_ERR_UNSUPPORTED;
+    case LAKE_PREC_AUTO: *prec = (n >= LAKE_AUTO_TC_MIN_N) ? 0 : -1; break;
+    default: return LAKE_ERR_INVAL;
+  }
+  return LAKE_OK;
+}
+
+int check_input_ptr(const void *in, int in_kind) {
+  const uintptr_t a = reinterpret_cast<uintptr_t>(in);
+  if (in_kind == LAKE_IN_RAW) return (a & 3) ? LAKE_ERR_INVAL : LAKE_OK;
+  return (a & 15) ? LAKE_ERR_INVAL : LAKE_OK;
+}
+
+struct ProfScope {
+  cudaStream_t s;
+  cudaEvent_t stop = nullptr;
+  explicit ProfScope(cudaStream_t st) : s(st) {
+    std::lock_guard<std::mutex> lk(g_prof_mu);
+    if (!g_prof) return;
+    if (g_prof_used == g_prof_ev.size()) {
+      cudaEvent_t a, b;
+      if (cudaEventCreate(&a) != cudaSuccess) return;
+      if (cudaEventCreate(&b) != cudaSuccess) { cudaEventDestroy(a); return; }
+      g_prof_ev.emplace_back(a, b);
+    }
+    auto &pr = g_prof_ev[g_prof_used++];
+    cudaEventRecord(pr.first, s);
+    stop = pr.second;
+  }
+  ~ProfScope() {
+    if (stop) cudaEventRecord(stop, s);
+  }
+};
+
+int launch_main(const void *in, int in_kind, int prec, const TileSched &ts, int nh_layout,
+                uint8_t *decisions, float *logits, cudaStream_t s, int device) {
+  cudaError_t e;
+  {
+    ProfScope ps(s);
+    if (prec < 0)
+      e = launch_mlp_fp32(in, in_kind, ts, decisions, logits, s, device);
+    else
+      e = launch_mlp_tc(in, in_kind, prec, ts, nh_layout, decisions, logits, s, device);
+  }
+  return cuda_status(e);
+}
+
+}  // namespace
+}  // namespace lake
+
+using namespace lake;
+
+extern "C" {
+
+size_t lake_linnos_blob_floats(int32_t arch) { return blob_floats(arch); }
+
+int lake_linnos_load_weights(int32_t model_id, int32_t arch, const float *blob, size_t n_floats,
+                             int32_t device) {
+  if (model_id < 0 || model_id >= LAKE_MAX_MODELS) return LAKE_ERR_INVAL;
+  if (arch < LAKE_ARCH_NN || arch > LAKE_ARCH_NN2) return LAKE_ERR_INVAL;
+  if (!blob || n_floats != blob_floats(arch)) return LAKE_ERR_INVAL;
+  if (device < 0 || device >= kMaxDevices) return LAKE_ERR_INVAL;
+  for (size_t i = 0; i < n_floats; ++i)
+    if (!std::isfinite(blob[i])) return LAKE_ERR_INVAL;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess) return LAKE_ERR_CUDA;
+  if (device >= ndev) return LAKE_ERR_INVAL;
+
+  const BlobView v = view_blob(arch, blob);
+  const int nh = v.nh;
+  // FP32 image: permuted W^T per hidden layer, biases, Wout, bout.
+  const size_t f_w0 = 32 * 256, f_wh = 256 * 256;
+  const size_t f_total = f_w0 + (nh - 1) * f_wh + nh * 256 + 2 * 256 + 4;
+  std::vector<float> f(f_total, 0.0f);
+  size_t off_wt[kMaxHiddenLayers], off_b[kMaxHiddenLayers], off_wout, off_bout;
+  {
+    size_t p = 0;
+    off_wt[0] = p;
+    for (int k = 0; k < 31; ++k)
+      for (int j = 0; j < 256; ++j) f[p + (size_t)k * 256 + perm_col(j)] = v.W[0][(size_t)j * 31 + k];
+    p += f_w0;
+    for (int l = 1; l < nh; ++l) {
+      off_wt[l] = p;
+      for (int k = 0; k < 256; ++k)
+        for (int j = 0; j < 256; ++j)
+          f[p + (size_t)k * 256 + perm_col(j)] = v.W[l][(size_t)j * 256 + k];
+      p += f_wh;
+    }
+    for (int l = 0; l < nh; ++l) {
+      off_b[l] = p;
+      std::memcpy(&f[p], v.b[l], 256 * 4);
+      p += 256;
+    }
+    off_wout = p;
+    std::memcpy(&f[p], v.W[nh], 512 * 4);
+    p += 512;
+    off_bout = p;
+    f[p] = v.b[nh][0];
+    f[p + 1] = v.b[nh][1];
+  }
+  const size_t tc_bytes = tc_image_bytes(nh);
+  std::vector<uint8_t> img(4 * tc_bytes);  // [prec][rank]
+  build_tc_image<__half>(v, img.data(), tc_bytes);
+  build_tc_image<__nv_bfloat16>(v, img.data() + 2 * tc_bytes, tc_bytes);
+
+  std::lock_guard<std::mutex> lk(g_mu);
+  DeviceGuard dg(device);
+  if (!dg.ok) return LAKE_ERR_CUDA;
+  DeviceState *st = nullptr;
+  int rc = get_state(device, &st);
+  if (rc != LAKE_OK) return rc;
+  ModelBufs nb;
+  if (cudaMalloc(&nb.fp32, f_total * 4) != cudaSuccess) return LAKE_ERR_NOMEM;
+  if (cudaMalloc(&nb.tc, img.size()) != cudaSuccess) {
+    free_bufs(nb);
+    return LAKE_ERR_NOMEM;
+  }
+  if (cudaMemcpy(nb.fp32, f.data(), f_total * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+      cudaMemcpy(nb.tc, img.data(), img.size(), cudaMemcpyHostToDevice) != cudaSuccess) {
+    free_bufs(nb);
+    return LAKE_ERR_CUDA;
+  }
+  DevModel m;
+  std::memset(&m, 0, sizeof(m));
+  m.arch = arch;
+  m.nh = nh;
+  m.tc_img[0] = static_cast<const uint8_t *>(nb.tc);
+  m.tc_img[1] = static_cast<const uint8_t *>(nb.tc) + 2 * tc_bytes;
+  m.tc_img_bytes = (uint32_t)tc_bytes;
+  const float *fb = static_cast<const float *>(nb.fp32);
+  for (int l = 0; l < nh; ++l) {
+    m.wt[l] = fb + off_wt[l];
+    m.b[l] = fb + off_b[l];
+  }
+  m.wout = fb + off_wout;
+  m.bout = fb + off_bout;
+  // publish: device table entry, then host mirror; free the previous buffers
+  if (cudaDeviceSynchronize() != cudaSuccess ||
+      cudaMemcpy(st->table + model_id, &m, sizeof(m), cudaMemcpyHostToDevice) != cudaSuccess) {
+    free_bufs(nb);
+    return LAKE_ERR_CUDA;
+  }
+  free_bufs(st->bufs[model_id]);
+  st->bufs[model_id] = nb;
+  st->host[model_id] = m;
+  return LAKE_OK;
+}
+
+int lake_linnos_unload(int32_t model_id, int32_t device) {
+  if (model_id < 0 || model_id >= LAKE_MAX_MODELS) return LAKE_ERR_INVAL;
+  if (device < 0 || device >= kMaxDevices) return LAKE_ERR_INVAL;
+  std::lock_guard<std::mutex> lk(g_mu);
+  DeviceState *st = g_dev[device];
+  if (!st || !st->init || st->host[model_id].arch < 0) return LAKE_ERR_NOMODEL;
+  DeviceGuard dg(device);
+  if (!dg.ok) return LAKE_ERR_CUDA;
+  DevModel m;
+  std::memset(&m, 0, sizeof(m));
+  m.arch = -1;
+  if (cudaDeviceSynchronize() != cudaSuccess ||
+      cudaMemcpy(st->table + model_id, &m, sizeof(m), cudaMemcpyHostToDevice) != cudaSuccess)
+    return LAKE_ERR_CUDA;
+  free_bufs(st->bufs[model_id]);
+  st->host[model_id] = m;
+  return LAKE_OK;
+}
+
+int lake_linnos_model_arch(int32_t model_id, int32_t device, int32_t *arch_out) {
+  if (!arch_out) return LAKE_ERR_INVAL;
+  if (model_id < 0 || model_id >= LAKE_MAX_MODELS) return LAKE_ERR_NOMODEL;
+  if (device < 0 || device >= kMaxDevices) return LAKE_ERR_INVAL;
+  std::lock_guard<std::mutex> lk(g_mu);
+  DeviceState *st = g_dev[device];
+  if (!st || st->host[model_id].arch < 0) return LAKE_ERR_NOMODEL;
+  *arch_out = st->host[model_id].arch;
+  return LAKE_OK;
+}
+
+int lake_linnos_digitize(const lake_io_raw_t *raw, int64_t n, uint8_t *digits, void *stream) {
+  if (n < 0) return LAKE_ERR_INVAL;
+  if (n == 0) return LAKE_OK;
+  if (!raw || !digits) return LAKE_ERR_INVAL;
+  if (reinterpret_cast<uintptr_t>(raw) & 3) return LAKE_ERR_INVAL;
+  return cuda_status(launch_digitize(raw, n, digits, static_cast<cudaStream_t>(stream)));
+}
+
+int lake_linnos_infer(const void *in, uint32_t flags, int64_t n, int32_t model_id,
+                      uint8_t *decisions, float *logits, void *stream) {
+  if (n < 0) return LAKE_ERR_INVAL;
+  int in_kind, prec;
+  int rc = check_flags(flags, n, &in_kind, &prec);
+  if (rc != LAKE_OK) return rc;
+  if (n == 0) return LAKE_OK;
+  if (!in || !decisions) return LAKE_ERR_INVAL;
+  if (check_input_ptr(in, in_kind) != LAKE_OK) return LAKE_ERR_INVAL;
+  if (logits && (reinterpret_cast<uintptr_t>(logits) & 3)) return LAKE_ERR_INVAL;
+  if (n > (int64_t)INT32_MAX) return LAKE_ERR_INVAL;
+  int device;
+  DevModel m;
+  rc = current_model(model_id, &device, &m, nullptr);
+  if (rc != LAKE_OK) return rc;
+  TileSched ts;
+  std::memset(&ts, 0, sizeof(ts));
+  const int rows = prec < 0 ? kF32TileM : kTcTileRows;
+  ts.n_tiles = (n + rows - 1) / rows;
+  ts.n = n;
+  ts.model = m;
+  return launch_main(in, in_kind, prec, ts, m.nh, decisions, logits,
+                     static_cast<cudaStream_t>(stream), device);
+}
+
+size_t lake_linnos_workspace_bytes(int64_t n) {
+  if (n < 0) return 0;
+  return group_workspace_bytes(n);
+}
+
+int lake_linnos_multi_group(int64_t n, const int32_t *model_ids, void *workspace,
+                            size_t ws_bytes, void *stream) {
+  if (n < 0 || n > (int64_t)INT32_MAX) return LAKE_ERR_INVAL;
+  if (n > 0 && !model_ids) return LAKE_ERR_INVAL;
+  if (!workspace) return LAKE_ERR_INVAL;
+  if (ws_bytes < group_workspace_bytes(n)) return LAKE_ERR_NOMEM;
+  int device, any;
+  const DevModel *table;
+  int rc = current_table(&device, &table, &any);
+  if (rc != LAKE_OK) return rc;
+  if (!table) {
+    // no model was ever loaded on this device: create the (empty) table so that every
+    // id is reported unknown
+    std::lock_guard<std::mutex> lk(g_mu);
+    DeviceState *st;
+    rc = get_state(device, &st);
+    if (rc != LAKE_OK) return rc;
+    table = st->table;
+  }
+  return cuda_status(
+      launch_group(n, model_ids, table, workspace, 0, static_cast<cudaStream_t>(stream)));
+}
+
+int lake_linnos_multi_grouped(const void *in, uint32_t flags, int64_t n, uint8_t *decisions,
+                              float *logits, void *workspace, size_t ws_bytes, void *stream) {
+  if (n < 0 || n > (int64_t)INT32_MAX) return LAKE_ERR_INVAL;
+  int in_kind, prec;
+  int rc = check_flags(flags, n, &in_kind, &prec);
+  if (rc != LAKE_OK) return rc;
+  if (n == 0) return LAKE_OK;
+  if (!in || !decisions || !workspace) return LAKE_ERR_INVAL;
+  if (check_input_ptr(in, in_kind) != LAKE_OK) return LAKE_ERR_INVAL;
+  if (ws_bytes < group_workspace_bytes(n)) return LAKE_ERR_NOMEM;
+  int device, any;
+  const DevModel *table;
+  rc = current_table(&device, &table, &any);
+  if (rc != LAKE_OK) return rc;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  cudaError_t e = launch_unknown_fill(workspace, n, decisions, logits, s);
+  if (e != cudaSuccess) return cuda_status(e);
+  if (!table || !any) return LAKE_OK;
+  TileSched ts;
+  std::memset(&ts, 0, sizeof(ts));
+  group_sched(workspace, n, prec < 0 ? 0 : 1, table, &ts);
+  return launch_main(in, in_kind, prec, ts, 3, decisions, logits, s, device);
+}
+
+int lake_linnos_infer_multi(const void *in, uint32_t flags, int64_t n, const int32_t *model_ids,
+                            uint8_t *decisions, float *logits, void *workspace, size_t ws_bytes,
+                            void *stream) {
+  if (n < 0) return LAKE_ERR_INVAL;
+  int in_kind, prec;
+  int rc = check_flags(flags, n, &in_kind, &prec);
+  if (rc != LAKE_OK) return rc;
+  if (n == 0) return LAKE_OK;
+  if (!in || !decisions || !model_ids || !workspace) return LAKE_ERR_INVAL;
+  if (check_input_ptr(in, in_kind) != LAKE_OK) return LAKE_ERR_INVAL;
+  rc = lake_linnos_multi_group(n, model_ids, workspace, ws_bytes, stream);
+  if (rc != LAKE_OK) return rc;
+  return lake_linnos_multi_grouped(in, flags, n, decisions, logits, workspace, ws_bytes, stream);
+}
+
+int lake_linnos_multi_status(const void *workspace, size_t ws_bytes, int64_t *n_unknown,
+                             void *stream) {
+  if (!workspace || !n_unknown) return LAKE_ERR_INVAL;
+  (void)ws_bytes;
+  GroupView v = group_view(const_cast<void *>(workspace), 0);
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  cudaError_t e = cudaMemcpyAsync(n_unknown, v.n_unknown, sizeof(int64_t),
+                                  cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  return cuda_status(e);
+}
+
+size_t lake_linnos_host_staging_bytes(int64_t n, uint32_t flags) {
+  if (n < 0) return 0;
+  const size_t in_b = (flags & LAKE_IN_MASK) == LAKE_IN_RAW ? 36 : 32;
+  auto a = [](size_t x) { return (x + 255) & ~(size_t)255; };
+  return a((size_t)n * in_b) + a((size_t)n * 4) + a((size_t)n) + a((size_t)n * 8) +
+         a(group_workspace_bytes(n));
+}
+
+int lake_linnos_infer_host(const void *h_in, uint32_t flags, int64_t n, int32_t model_id,
+                           const int32_t *h_model_ids, uint8_t *h_decisions, float *h_logits,
+                           void *d_staging, size_t staging_bytes, void *stream) {
+  if (n < 0) return LAKE_ERR_INVAL;
+  int in_kind, prec;
+  int rc = check_flags(flags, n, &in_kind, &prec);
+  if (rc != LAKE_OK) return rc;
+  if (n == 0) return LAKE_OK;
+  if (!h_in || !h_decisions || !d_staging) return LAKE_ERR_INVAL;
+  if (staging_bytes < lake_linnos_host_staging_bytes(n, flags)) return LAKE_ERR_NOMEM;
+  auto a = [](size_t x) { return (x + 255) & ~(size_t)255; };
+  const size_t in_b = in_kind == LAKE_IN_RAW ? 36 : 32;
+  uint8_t *p = static_cast<uint8_t *>(d_staging);
+  void *d_in = p; p += a((size_t)n * in_b);
+  int32_t *d_ids = reinterpret_cast<int32_t *>(p); p += a((size_t)n * 4);
+  uint8_t *d_dec = p; p += a((size_t)n);
+  float *d_log = reinterpret_cast<float *>(p); p += a((size_t)n * 8);
+  void *d_ws = p;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  cudaError_t e = cudaMemcpyAsync(d_in, h_in, (size_t)n * in_b, cudaMemcpyHostToDevice, s);
+  if (e != cudaSuccess) return cuda_status(e);
+  if (h_model_ids) {
+    e = cudaMemcpyAsync(d_ids, h_model_ids, (size_t)n * 4, cudaMemcpyHostToDevice, s);
+    if (e != cudaSuccess) return cuda_status(e);
+    rc = lake_linnos_infer_multi(d_in, flags, n, d_ids, d_dec, h_logits ? d_log : nullptr,
+                                 d_ws, a(group_workspace_bytes(n)), stream);
+  } else {
+    rc = lake_linnos_infer(d_in, flags, n, model_id, d_dec, h_logits ? d_log : nullptr, stream);
+  }
+  if (rc != LAKE_OK) return rc;
+  e = cudaMemcpyAsync(h_decisions, d_dec, (size_t)n, cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess && h_logits)
+    e = cudaMemcpyAsync(h_logits, d_log, (size_t)n * 8, cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  return cuda_status(e);
+}
+
+uint64_t lake_linnos_launch_count(void) { return g_launches.load(); }
+void lake_linnos_reset_launch_count(void) { g_launches.store(0); }
+
+int lake_linnos_profile_enable(int enable) {
+  std::lock_guard<std::mutex> lk(g_prof_mu);
+  g_prof = enable != 0;
+  g_prof_used = 0;
+  return LAKE_OK;
+}
+
+int lake_linnos_profile_read(double *total_ms, int64_t *n_launches) {
+  if (!total_ms || !n_launches) return LAKE_ERR_INVAL;
+  std::lock_guard<std::mutex> lk(g_prof_mu);
+  double tot = 0.0;
+  for (size_t i = 0; i < g_prof_used; ++i) {
+    cudaError_t e = cudaEventSynchronize(g_prof_ev[i].second);
+    if (e != cudaSuccess) return cuda_status(e);
+    float ms = 0.0f;
+    e = cudaEventElapsedTime(&ms, g_prof_ev[i].first, g_prof_ev[i].second);
+    if (e != cudaSuccess) return cuda_status(e);
+    tot += ms;
+  }
+  *total_ms = tot;
+  *n_launches = (int64_t)g_prof_used;
+  g_prof_used = 0;
+  return LAKE_OK;
+}
+
+const char *lake_linnos_strerror(int status) {
+  switch (status) {
+    case LAKE_OK: return "ok";
+    case LAKE_ERR_INVAL: return "invalid argument";
+    case LAKE_ERR_NOMODEL: return "model not loaded on the current device";
+    case LAKE_ERR_CUDA: return "CUDA error";
+    case LAKE_ERR_NOMEM: return "out of memory or workspace too small";
+    case LAKE_ERR_UNSUPPORTED: return "unsupported in this build";
+    default: return "unknown status";
+  }
+}
+
+}  // extern "C"

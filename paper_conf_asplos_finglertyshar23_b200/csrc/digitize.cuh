@@ -1,0 +1,48 @@
+// digitize.cuh — device-side digitisation of one raw I/O record (product path).
+//
+// Definition (BASELINE.json north_star; readings R1-R6 in DESIGN.md §3): the 31 LinnOS
+// inputs are D3(q_now) | D4(lat_us[0..3]) | D3(q_hist[0..3]), where Dw(v) is the w
+// decimal digits of min(v, 10^w - 1), most significant first. Feature semantics: PAPER.md
+// §5.5, §7.1; history index 0 = most recent, §5.2 P:769-772.
+//
+// Integer only, so it is bit-exact by construction; the caller chooses what to do with the
+// digits (bytes for lake_linnos_digitize, fp32 / fp16 / bf16 operands inside the fused
+// kernels). Division by a constant compiles to multiply-high.
+#pragma once
+#include <cstdint>
+
+namespace lake {
+
+// Emit the w digits of min(v, 10^w-1) MSB-first through f(position, digit).
+template <int W, typename F>
+__device__ __forceinline__ void emit_digits(uint32_t v, int pos, F &&f) {
+  constexpr uint32_t cap = (W == 3) ? 999u : 9999u;
+  uint32_t m = v < cap ? v : cap;
+  if constexpr (W == 4) {
+    uint32_t d0 = m / 1000u;
+    uint32_t r = m - d0 * 1000u;
+    uint32_t d1 = r / 100u;
+    r -= d1 * 100u;
+    uint32_t d2 = r / 10u;
+    uint32_t d3 = r - d2 * 10u;
+    f(pos + 0, d0); f(pos + 1, d1); f(pos + 2, d2); f(pos + 3, d3);
+  } else {
+    uint32_t d0 = m / 100u;
+    uint32_t r = m - d0 * 100u;
+    uint32_t d1 = r / 10u;
+    uint32_t d2 = r - d1 * 10u;
+    f(pos + 0, d0); f(pos + 1, d1); f(pos + 2, d2);
+  }
+}
+
+// rec = {q_now, lat_us[0..3], q_hist[0..3]}; f(position 0..30, digit 0..9).
+template <typename F>
+__device__ __forceinline__ void digitize_record(const uint32_t (&rec)[9], F &&f) {
+  emit_digits<3>(rec[0], 0, f);
+#pragma unroll
+  for (int k = 0; k < 4; ++k) emit_digits<4>(rec[1 + k], 3 + 4 * k, f);
+#pragma unroll
+  for (int k = 0; k < 4; ++k) emit_digits<3>(rec[5 + k], 19 + 3 * k, f);
+}
+
+}  // namespace lake

@@ -1,0 +1,305 @@
+// group.cu — model grouping for lake_linnos_infer_multi: one feature registry (hence one
+// model) per block device (Fig. 4 caption); batches from several
+// devices arrive interleaved and are scored per model (score_features).
+//
+// Counting sort of I/O indices by model id, on the device:
+//   group_hist     per-block SMEM histogram -> one global atomic per (block, model)
+//   group_scan     one block: exclusive scans of counts and of tiles per model (for both
+//                  the 64-row FP32 tiles and the 256-row tensor-core tiles)
+//   group_scatter  per-block SMEM histogram -> reserve a range per model -> positions
+//   group_tiles    one thread per tile: binary search of its model, begin, count
+// Unknown ids (out of range or not loaded) go to the tail of perm; lake_linnos_multi_grouped
+// writes decision 0 / NaN logits for them. Results do not depend on the order inside a
+// model's range (every row is computed independently), so the scatter need not be stable.
+#include "lake_internal.h"
+
+namespace lake {
+namespace {
+
+constexpr int kGBlock = 512;
+constexpr int kChunk = 8192;  // I/Os per block-iteration in hist/scatter
+
+struct WsHeader {
+  int32_t counts[LAKE_MAX_MODELS];
+  int32_t cursor[LAKE_MAX_MODELS];
+  int32_t offsets[LAKE_MAX_MODELS];
+  int32_t tile_off64[LAKE_MAX_MODELS + 1];
+  int32_t tile_off256[LAKE_MAX_MODELS + 1];
+  int32_t n_tiles64;
+  int32_t n_tiles256;
+  int32_t n_known;
+  int32_t unk_cursor;
+  int64_t n_unknown;
+  int32_t arch_mask;
+  int32_t pad;
+};
+
+__host__ __device__ inline size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
+
+struct WsLayout {
+  size_t header, perm, t64_model, t64_begin, t64_count, t256_model, t256_begin, t256_count,
+      total;
+  int64_t max64, max256;
+};
+
+WsLayout ws_layout(int64_t n) {
+  WsLayout L{};
+  L.max64 = group_max_tiles(n, kF32TileM);
+  L.max256 = group_max_tiles(n, kTcTileRows);
+  size_t off = 0;
+  L.header = off; off = align256(off + sizeof(WsHeader));
+  L.perm = off; off = align256(off + (size_t)n * 4);
+  L.t64_model = off; off = align256(off + (size_t)L.max64 * 4);
+  L.t64_begin = off; off = align256(off + (size_t)L.max64 * 8);
+  L.t64_count = off; off = align256(off + (size_t)L.max64 * 4);
+  L.t256_model = off; off = align256(off + (size_t)L.max256 * 4);
+  L.t256_begin = off; off = align256(off + (size_t)L.max256 * 8);
+  L.t256_count = off; off = align256(off + (size_t)L.max256 * 4);
+  L.total = off;
+  return L;
+}
+
+__device__ __forceinline__ bool known(const DevModel *table, int32_t m) {
+  return m >= 0 && m < LAKE_MAX_MODELS && table[m].arch >= 0;
+}
+
+__global__ void __launch_bounds__(kGBlock)
+group_hist(const int32_t *__restrict__ ids, int64_t n, const DevModel *__restrict__ table,
+           WsHeader *h) {
+  __shared__ int32_t cnt[LAKE_MAX_MODELS + 1];
+  for (int64_t base = (int64_t)blockIdx.x * kChunk; base < n; base += (int64_t)gridDim.x * kChunk) {
+    for (int i = threadIdx.x; i <= LAKE_MAX_MODELS; i += kGBlock) cnt[i] = 0;
+    __syncthreads();
+    const int64_t end = (base + kChunk) < n ? base + kChunk : n;
+    for (int64_t i = base + threadIdx.x; i < end; i += kGBlock) {
+      const int32_t m = __ldg(ids + i);
+      atomicAdd(&cnt[known(table, m) ? m : LAKE_MAX_MODELS], 1);
+    }
+    __syncthreads();
+    for (int m = threadIdx.x; m < LAKE_MAX_MODELS; m += kGBlock)
+      if (cnt[m]) atomicAdd(&h->counts[m], cnt[m]);
+    if (threadIdx.x == 0 && cnt[LAKE_MAX_MODELS])
+      atomicAdd((unsigned long long *)&h->n_unknown, (unsigned long long)cnt[LAKE_MAX_MODELS]);
+    __syncthreads();
+  }
+}
+
+// exclusive block scan over 1024 values (1024 threads)
+__device__ int32_t block_excl_scan(int32_t v, int32_t *warp_tot, int32_t *total) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  int32_t x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int32_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) warp_tot[w] = x;
+  __syncthreads();
+  if (w == 0) {
+    int32_t t = warp_tot[lane];
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int32_t y = __shfl_up_sync(0xffffffffu, t, o);
+      if (lane >= o) t += y;
+    }
+    warp_tot[lane] = t;  // inclusive over warps
+    if (lane == 31) *total = t;
+  }
+  __syncthreads();
+  const int32_t r = x - v + (w > 0 ? warp_tot[w - 1] : 0);
+  __syncthreads();
+  return r;
+}
+
+__global__ void __launch_bounds__(LAKE_MAX_MODELS)
+group_scan(WsHeader *h) {
+  __shared__ int32_t warp_tot[32];
+  __shared__ int32_t total;
+  const int m = threadIdx.x;
+  const int32_t c = h->counts[m];
+  const int32_t off = block_excl_scan(c, warp_tot, &total);
+  h->offsets[m] = off;
+  h->cursor[m] = off;
+  const int32_t n_known = total;
+  const int32_t t64 = block_excl_scan((c + kF32TileM - 1) / kF32TileM, warp_tot, &total);
+  h->tile_off64[m] = t64;
+  const int32_t tot64 = total;
+  const int32_t t256 = block_excl_scan((c + kTcTileRows - 1) / kTcTileRows, warp_tot, &total);
+  h->tile_off256[m] = t256;
+  if (m == 0) {
+    h->n_known = n_known;
+    h->unk_cursor = n_known;
+    h->n_tiles64 = tot64;
+    h->n_tiles256 = total;
+    h->tile_off64[LAKE_MAX_MODELS] = tot64;
+    h->tile_off256[LAKE_MAX_MODELS] = total;
+  }
+}
+
+__global__ void __launch_bounds__(kGBlock)
+group_scatter(const int32_t *__restrict__ ids, int64_t n, const DevModel *__restrict__ table,
+              WsHeader *h, int32_t *__restrict__ perm) {
+  __shared__ int32_t cnt[LAKE_MAX_MODELS + 1];
+  __shared__ int32_t basep[LAKE_MAX_MODELS + 1];
+  for (int64_t base = (int64_t)blockIdx.x * kChunk; base < n; base += (int64_t)gridDim.x * kChunk) {
+    for (int i = threadIdx.x; i <= LAKE_MAX_MODELS; i += kGBlock) cnt[i] = 0;
+    __syncthreads();
+    const int64_t end = (base + kChunk) < n ? base + kChunk : n;
+    for (int64_t i = base + threadIdx.x; i < end; i += kGBlock) {
+      const int32_t m = __ldg(ids + i);
+      atomicAdd(&cnt[known(table, m) ? m : LAKE_MAX_MODELS], 1);
+    }
+    __syncthreads();
+    for (int m = threadIdx.x; m <= LAKE_MAX_MODELS; m += kGBlock) {
+      const int32_t c = cnt[m];
+      if (c) basep[m] = atomicAdd(m < LAKE_MAX_MODELS ? &h->cursor[m] : &h->unk_cursor, c);
+      cnt[m] = 0;
+    }
+    __syncthreads();
+    for (int64_t i = base + threadIdx.x; i < end; i += kGBlock) {
+      const int32_t m0 = __ldg(ids + i);
+      const int32_t m = known(table, m0) ? m0 : LAKE_MAX_MODELS;
+      const int32_t r = atomicAdd(&cnt[m], 1);
+      perm[basep[m] + r] = (int32_t)i;
+    }
+    __syncthreads();
+  }
+}
+
+__device__ __forceinline__ int find_model(const int32_t *off, int32_t t) {
+  int lo = 0, hi = LAKE_MAX_MODELS;  // off[lo] <= t < off[hi]
+  while (hi - lo > 1) {
+    const int mid = (lo + hi) >> 1;
+    if (off[mid] <= t) lo = mid; else hi = mid;
+  }
+  return lo;
+}
+
+__global__ void group_tiles(const WsHeader *__restrict__ h, int64_t max64, int64_t max256,
+                            int32_t *t64_model, int64_t *t64_begin, int32_t *t64_count,
+                            int32_t *t256_model, int64_t *t256_begin, int32_t *t256_count) {
+  const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (t < h->n_tiles64 && t < max64) {
+    const int m = find_model(h->tile_off64, (int32_t)t);
+    const int32_t local = (int32_t)t - h->tile_off64[m];
+    const int32_t rem = h->counts[m] - local * kF32TileM;
+    t64_model[t] = m;
+    t64_begin[t] = (int64_t)h->offsets[m] + (int64_t)local * kF32TileM;
+    t64_count[t] = rem < kF32TileM ? rem : kF32TileM;
+  }
+  if (t < h->n_tiles256 && t < max256) {
+    const int m = find_model(h->tile_off256, (int32_t)t);
+    const int32_t local = (int32_t)t - h->tile_off256[m];
+    const int32_t rem = h->counts[m] - local * kTcTileRows;
+    t256_model[t] = m;
+    t256_begin[t] = (int64_t)h->offsets[m] + (int64_t)local * kTcTileRows;
+    t256_count[t] = rem < kTcTileRows ? rem : kTcTileRows;
+  }
+}
+
+__global__ void unknown_fill(const WsHeader *__restrict__ h, int64_t n,
+                             const int32_t *__restrict__ perm, uint8_t *decisions,
+                             float *logits) {
+  const int64_t start = h->n_known;
+  for (int64_t p = start + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < n;
+       p += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t io = perm[p];
+    decisions[io] = 0;
+    if (logits) {
+      logits[(int64_t)io * 2] = __int_as_float(0x7fc00000);
+      logits[(int64_t)io * 2 + 1] = __int_as_float(0x7fc00000);
+    }
+  }
+}
+
+}  // namespace
+
+int64_t group_max_tiles(int64_t n, int tile_rows) {
+  return (n + tile_rows - 1) / tile_rows + LAKE_MAX_MODELS;
+}
+
+size_t group_workspace_bytes(int64_t n) { return ws_layout(n).total; }
+
+GroupView group_view(void *ws, int64_t n) {
+  const WsLayout L = ws_layout(n);
+  uint8_t *b = static_cast<uint8_t *>(ws);
+  WsHeader *h = reinterpret_cast<WsHeader *>(b + L.header);
+  GroupView v{};
+  v.perm = reinterpret_cast<int32_t *>(b + L.perm);
+  v.n_unknown = &h->n_unknown;
+  v.counts = h->counts;
+  return v;
+}
+
+struct GroupPtrs {
+  WsHeader *h;
+  int32_t *perm;
+  int32_t *tm[2];
+  int64_t *tb[2];
+  int32_t *tc[2];
+  int32_t *nt[2];
+  int64_t max[2];
+};
+
+static GroupPtrs group_ptrs(void *ws, int64_t n) {
+  const WsLayout L = ws_layout(n);
+  uint8_t *b = static_cast<uint8_t *>(ws);
+  GroupPtrs p{};
+  p.h = reinterpret_cast<WsHeader *>(b + L.header);
+  p.perm = reinterpret_cast<int32_t *>(b + L.perm);
+  p.tm[0] = reinterpret_cast<int32_t *>(b + L.t64_model);
+  p.tb[0] = reinterpret_cast<int64_t *>(b + L.t64_begin);
+  p.tc[0] = reinterpret_cast<int32_t *>(b + L.t64_count);
+  p.tm[1] = reinterpret_cast<int32_t *>(b + L.t256_model);
+  p.tb[1] = reinterpret_cast<int64_t *>(b + L.t256_begin);
+  p.tc[1] = reinterpret_cast<int32_t *>(b + L.t256_count);
+  p.nt[0] = &p.h->n_tiles64;
+  p.nt[1] = &p.h->n_tiles256;
+  p.max[0] = L.max64;
+  p.max[1] = L.max256;
+  return p;
+}
+
+cudaError_t launch_group(int64_t n, const int32_t *model_ids, const DevModel *table, void *ws,
+                         int /*tile_rows*/, cudaStream_t s) {
+  GroupPtrs p = group_ptrs(ws, n);
+  cudaError_t e = cudaMemsetAsync(p.h, 0, sizeof(WsHeader), s);
+  if (e != cudaSuccess) return e;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int64_t chunks = (n + kChunk - 1) / kChunk;
+  const int grid = (int)(chunks < 2 * sms ? chunks : 2 * sms);
+  if (grid > 0) group_hist<<<grid, kGBlock, 0, s>>>(model_ids, n, table, p.h);
+  group_scan<<<1, LAKE_MAX_MODELS, 0, s>>>(p.h);
+  if (grid > 0) group_scatter<<<grid, kGBlock, 0, s>>>(model_ids, n, table, p.h, p.perm);
+  const int64_t mt = p.max[0] > p.max[1] ? p.max[0] : p.max[1];
+  group_tiles<<<(unsigned)((mt + 255) / 256), 256, 0, s>>>(p.h, p.max[0], p.max[1], p.tm[0],
+                                                           p.tb[0], p.tc[0], p.tm[1], p.tb[1],
+                                                           p.tc[1]);
+  count_launch(grid > 0 ? 4 : 2);
+  return cudaGetLastError();
+}
+
+// Fill a TileSched for the grouped launch; which = 0 (64-row FP32 tiles) / 1 (256-row TC).
+void group_sched(void *ws, int64_t n, int which, const DevModel *table, TileSched *ts) {
+  GroupPtrs p = group_ptrs(ws, n);
+  ts->tile_model = p.tm[which];
+  ts->tile_begin = p.tb[which];
+  ts->tile_count = p.tc[which];
+  ts->perm = p.perm;
+  ts->n_tiles_dev = p.nt[which];
+  ts->n_tiles = p.max[which];
+  ts->n = n;
+  ts->table = table;
+}
+
+cudaError_t launch_unknown_fill(void *ws, int64_t n, uint8_t *decisions, float *logits,
+                                cudaStream_t s) {
+  GroupPtrs p = group_ptrs(ws, n);
+  unknown_fill<<<64, 256, 0, s>>>(p.h, n, p.perm, decisions, logits);
+  count_launch();
+  return cudaGetLastError();
+}
+
+}  // namespace lake

@@ -1,0 +1,95 @@
+// lake_internal.h — internal types shared by the C-ABI layer (api.cu) and the kernels.
+// Not part of the public ABI (include/lake_linnos.h is).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "../../include/lake_linnos.h"
+
+namespace lake {
+
+constexpr int kHidden = 256;
+constexpr int kInputs = 31;
+constexpr int kMaxHiddenLayers = 3;
+
+// ---- FP32 CUDA-core path (mlp_fp32.cu) ------------------------------------------------
+// Per layer l the weights are stored transposed, W^T[k][j], k < K_l, with the 256 output
+// columns permuted so that thread tc's 8 columns {tc + 32*jj} are two contiguous float4
+// groups: position p(j) = (jj/4)*128 + tc*4 + (jj%4) with tc = j%32, jj = j/32.
+constexpr int kF32TileM = 64;       // I/Os per CTA tile
+constexpr int kF32Threads = 256;
+constexpr int kF32KChunk = 16;      // rows of W^T staged per pipeline stage
+constexpr int kF32ActStride = 68;   // floats per activation row in SMEM (64 + 4 pad)
+
+// ---- tcgen05 path (mlp_tc.cu) ------------------------------------------------------------
+// A CTA pair (cluster of 2, cta_group::2) processes a 256-row tile: each CTA owns 128 rows
+// of A and D, and holds half (N/2 rows) of every weight matrix, in the K-major SWIZZLE_NONE
+// UMMA layout: core matrix (8 rows x 16 B) for (row group rg, k group kg) at byte offset
+// kg * (R * 16) + rg * 128, i.e. LBO = R*16 bytes (K direction), SBO = 128 bytes.
+constexpr int kTcRowsPerCta = 128;
+constexpr int kTcTileRows = 256;
+constexpr int kTcK0 = 32;                                   // 31 digits + zero pad
+constexpr int kTcOutN = 16;                                 // 2 classes padded to N=16
+constexpr uint32_t kTcW0HalfBytes = 128 * kTcK0 * 2;        // 8 KB
+constexpr uint32_t kTcWhHalfBytes = 128 * kHidden * 2;      // 64 KB
+constexpr uint32_t kTcWoHalfBytes = (kTcOutN / 2) * kHidden * 2;  // 4 KB
+__host__ __device__ constexpr uint32_t tc_bias_floats(int nh) { return nh * kHidden + 4; }
+__host__ __device__ constexpr uint32_t tc_image_bytes(int nh) {
+  return kTcW0HalfBytes + (nh - 1) * kTcWhHalfBytes + kTcWoHalfBytes + tc_bias_floats(nh) * 4;
+}
+
+struct DevModel {
+  int32_t arch;      // -1 = slot empty
+  int32_t nh;        // hidden layers: 1, 2, 3
+  // tcgen05 images: [0]=fp16, [1]=bf16; each holds rank-0 half then rank-1 half.
+  const uint8_t *tc_img[2];
+  uint32_t tc_img_bytes;  // bytes per rank half
+  uint32_t pad0;
+  // FP32 path
+  const float *wt[kMaxHiddenLayers];  // permuted W^T; layer 0 is [32][256] (row 31 zero)
+  const float *b[kMaxHiddenLayers];
+  const float *wout;                  // [2][256]
+  const float *bout;                  // [2]
+};
+
+// Tile schedule. Single-model calls use tile_model == nullptr (all tiles -> `model`) and
+// implicit contiguous tiles; multi-model calls read a device-built grouping.
+struct TileSched {
+  const int32_t *tile_model;   // [n_tiles] model slot per tile, or nullptr
+  const int64_t *tile_begin;   // [n_tiles] first position in `perm`
+  const int32_t *tile_count;   // [n_tiles] rows in the tile
+  const int32_t *perm;         // position -> I/O index, or nullptr (identity)
+  const int32_t *n_tiles_dev;  // device tile count (multi) or nullptr
+  int64_t n_tiles;             // host tile count (single) / upper bound (multi)
+  int64_t n;                   // I/Os
+  const DevModel *table;       // device model table (multi)
+  DevModel model;              // single-model copy
+};
+
+// Kernel launchers (return cudaError_t of the launch).
+cudaError_t launch_digitize(const lake_io_raw_t *raw, int64_t n, uint8_t *digits,
+                            cudaStream_t s);
+cudaError_t launch_mlp_fp32(const void *in, int in_kind, const TileSched &ts,
+                            uint8_t *decisions, float *logits, cudaStream_t s, int device);
+cudaError_t launch_mlp_tc(const void *in, int in_kind, int prec, const TileSched &ts, int nh,
+                          uint8_t *decisions, float *logits, cudaStream_t s, int device);
+// Grouping for infer_multi (group.cu).
+size_t group_workspace_bytes(int64_t n);
+int64_t group_max_tiles(int64_t n, int tile_rows);
+cudaError_t launch_group(int64_t n, const int32_t *model_ids, const DevModel *table,
+                         void *ws, int tile_rows, cudaStream_t s);
+// which = 0: 64-row FP32 tiles, 1: 256-row tensor-core tiles
+void group_sched(void *ws, int64_t n, int which, const DevModel *table, TileSched *ts);
+cudaError_t launch_unknown_fill(void *ws, int64_t n, uint8_t *decisions, float *logits,
+                                cudaStream_t s);
+struct GroupView {
+  int32_t *perm;
+  int64_t *n_unknown;
+  int32_t *counts;
+};
+GroupView group_view(void *ws, int64_t n);
+size_t tc_smem_bytes(int nh_layout);
+
+void count_launch(int k = 1);
+
+}  // namespace lake

@@ -1,0 +1,208 @@
+// mlp_fp32.cu — fused digitise -> MLP -> argmax on CUDA cores in FP32, bit-exact with the
+// oracle under reading R15: every output accumulates from +0.0f with one
+// __fmaf_rn per input in ascending k, then one __fadd_rn of the bias, then ReLU as
+// (z > 0 ? z : +0). No split-K, no tree reduction, no FTZ, no contraction (--fmad=false).
+//
+// Network: "two layers with 256 and 2 neurons" (+1 / +2 hidden layers), §7.1
+// P:1168-1177. Batch scoring (score_features, Table 1).
+//
+// Mapping: a CTA (256 threads) owns a 64-I/O tile. Hidden layers are register-tiled GEMMs:
+// thread (tr = warp, tc = lane) owns 8 rows {tr*4+i, 32+tr*4+i} x 8 columns {tc + 32*jj}.
+// Each accumulator is summed over k strictly in order (that is what a K-loop GEMM does),
+// so the tiling changes nothing numerically. Activations live transposed in SMEM
+// (act[k][row], row stride 68 floats: broadcast A reads, conflict-free epilogue stores);
+// weights stream through a 2-stage cp.async pipeline in 16-row chunks of W^T whose columns
+// were permuted at load time so each thread's 8 columns are two float4s.
+// The 2-wide output layer is one sequential fmaf chain per (row, class).
+#include <cuda_pipeline.h>
+
+#include "digitize.cuh"
+#include "lake_internal.h"
+
+namespace lake {
+namespace {
+
+constexpr int M = kF32TileM;
+constexpr int S = kF32ActStride;
+constexpr int KC = kF32KChunk;
+
+struct F32Smem {
+  float act[2][kHidden][S];     // transposed activations, ping-pong
+  float w[2][KC][kHidden];      // W^T chunk staging (permuted columns)
+  float wout[2][kHidden];
+  float bout[4];
+  int32_t rows[M];              // I/O index per tile row, -1 = padding
+};
+
+__device__ __forceinline__ void stage_chunk(float (*dst)[kHidden], const float *src, int rows) {
+  // rows x 256 floats, contiguous in global; 16-byte cp.async per thread-iteration.
+  const int n16 = rows * kHidden / 4;
+  for (int i = threadIdx.x; i < n16; i += kF32Threads) {
+    __pipeline_memcpy_async(reinterpret_cast<float4 *>(&dst[0][0]) + i,
+                            reinterpret_cast<const float4 *>(src) + i, 16);
+  }
+  __pipeline_commit();
+}
+
+template <int IN_KIND>
+__global__ void __launch_bounds__(kF32Threads, 1)
+mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
+                uint8_t *__restrict__ decisions,
+                float *__restrict__ logits) {
+  extern __shared__ __align__(16) uint8_t smem_raw[];
+  F32Smem &sm = *reinterpret_cast<F32Smem *>(smem_raw);
+  const int tid = threadIdx.x;
+  const int tr = tid >> 5;   // warp: row group
+  const int tc = tid & 31;   // lane: column group
+  const int64_t n_tiles = ts.n_tiles_dev ? (int64_t)*ts.n_tiles_dev : ts.n_tiles;
+
+  for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
+    const DevModel *mp = ts.tile_model ? &ts.table[ts.tile_model[tile]] : &ts.model;
+    const int nh = mp->nh;
+    int64_t begin;
+    int count;
+    if (ts.tile_model) {
+      begin = ts.tile_begin[tile];
+      count = ts.tile_count[tile];
+    } else {
+      begin = tile * M;
+      count = (int)((ts.n - begin) < M ? (ts.n - begin) : M);
+    }
+    __syncthreads();  // previous tile's output layer is done with act[] / wout
+    // ---- rows, digits -> act[0][k][r] (k < 32, row 31 = 0) --------------------------
+    if (tid < M) {
+      int32_t io = -1;
+      if (tid < count) io = ts.perm ? ts.perm[begin + tid] : (int32_t)(begin + tid);
+      sm.rows[tid] = io;
+      float (*a0)[S] = sm.act[0];
+      if (io < 0) {
+        for (int k = 0; k < 32; ++k) a0[k][tid] = 0.0f;
+      } else if (IN_KIND == LAKE_IN_RAW) {
+        const uint32_t *r = reinterpret_cast<const uint32_t *>(in) + (int64_t)io * 9;
+        uint32_t rec[9];
+#pragma unroll
+        for (int f = 0; f < 9; ++f) rec[f] = __ldg(r + f);
+        digitize_record(rec, [&](int pos, uint32_t d) { a0[pos][tid] = (float)d; });
+        a0[31][tid] = 0.0f;
+      } else {
+        const uint4 *p = reinterpret_cast<const uint4 *>(
+            reinterpret_cast<const uint8_t *>(in) + (int64_t)io * 32);
+        uint4 v0 = __ldg(p), v1 = __ldg(p + 1);
+        uint32_t w[8] = {v0.x, v0.y, v0.z, v0.w, v1.x, v1.y, v1.z, v1.w};
+#pragma unroll
+        for (int k = 0; k < 32; ++k) a0[k][tid] = (float)((w[k >> 2] >> ((k & 3) * 8)) & 0xFFu);
+      }
+    } else if (tid < M + 2 * kHidden / 4 + 1) {
+      // output-layer weights for this tile's model
+      const int i = tid - M;
+      if (i < 2 * kHidden / 4)
+        reinterpret_cast<float4 *>(&sm.wout[0][0])[i] =
+            __ldg(reinterpret_cast<const float4 *>(mp->wout) + i);
+      else {
+        sm.bout[0] = __ldg(mp->bout);
+        sm.bout[1] = __ldg(mp->bout + 1);
+      }
+    }
+    // ---- hidden layers -----------------------------------------------------------------
+    for (int l = 0; l < nh; ++l) {
+      const int K = (l == 0) ? kInputs : kHidden;         // strict: layer 0 sums 31 terms
+      const int Kst = (l == 0) ? 32 : kHidden;            // staged rows (row 31 is zero)
+      const float *wt = mp->wt[l];
+      const float (*ain)[S] = sm.act[l & 1];
+      float (*aout)[S] = sm.act[(l + 1) & 1];
+      float acc[8][8];
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+#pragma unroll
+        for (int j = 0; j < 8; ++j) acc[i][j] = 0.0f;
+      const int nch = Kst / KC;
+      stage_chunk(sm.w[0], wt, KC);
+      for (int c = 0; c < nch; ++c) {
+        if (c + 1 < nch) {
+          stage_chunk(sm.w[(c + 1) & 1], wt + (int64_t)(c + 1) * KC * kHidden, KC);
+          __pipeline_wait_prior(1);
+        } else {
+          __pipeline_wait_prior(0);
+        }
+        __syncthreads();
+        const float (*wc)[kHidden] = sm.w[c & 1];
+        const int kmax = (K - c * KC) < KC ? (K - c * KC) : KC;
+#pragma unroll 4
+        for (int kk = 0; kk < kmax; ++kk) {
+          const int k = c * KC + kk;
+          const float4 a0 = *reinterpret_cast<const float4 *>(&ain[k][tr * 4]);
+          const float4 a1 = *reinterpret_cast<const float4 *>(&ain[k][32 + tr * 4]);
+          const float4 b0 = *reinterpret_cast<const float4 *>(&wc[kk][tc * 4]);
+          const float4 b1 = *reinterpret_cast<const float4 *>(&wc[kk][128 + tc * 4]);
+          const float av[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+          const float bv[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+#pragma unroll
+          for (int i = 0; i < 8; ++i)
+#pragma unroll
+            for (int j = 0; j < 8; ++j) acc[i][j] = __fmaf_rn(av[i], bv[j], acc[i][j]);
+        }
+        __syncthreads();
+      }
+      // epilogue: z = acc + b (one rounding), ReLU, store transposed
+      const float *bias = mp->b[l];
+#pragma unroll
+      for (int jj = 0; jj < 8; ++jj) {
+        const int j = tc + 32 * jj;
+        const float bj = __ldg(bias + j);
+        float h[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const float z = __fadd_rn(acc[i][jj], bj);
+          h[i] = (z > 0.0f) ? z : 0.0f;
+        }
+        *reinterpret_cast<float4 *>(&aout[j][tr * 4]) = make_float4(h[0], h[1], h[2], h[3]);
+        *reinterpret_cast<float4 *>(&aout[j][32 + tr * 4]) = make_float4(h[4], h[5], h[6], h[7]);
+      }
+      __syncthreads();
+    }
+    // ---- output layer (2 neurons, identity) + decision ------------------------------------
+    if (tid < 2 * M) {
+      const int r = tid >> 1, c = tid & 1;
+      const float (*h)[S] = sm.act[nh & 1];
+      float acc = 0.0f;
+#pragma unroll 8
+      for (int k = 0; k < kHidden; ++k) acc = __fmaf_rn(h[k][r], sm.wout[c][k], acc);
+      const float z = __fadd_rn(acc, sm.bout[c]);
+      const float other = __shfl_xor_sync(0xffffffffu, z, 1);
+      const int32_t io = sm.rows[r];
+      if (io >= 0) {
+        if (logits) logits[(int64_t)io * 2 + c] = z;
+        if (c == 0) decisions[io] = (other > z) ? 1 : 0;  // logit1 > logit0; ties/NaN -> 0
+      }
+    }
+  }
+}
+
+}  // namespace
+
+cudaError_t launch_mlp_fp32(const void *in, int in_kind, const TileSched &ts,
+                            uint8_t *decisions, float *logits, cudaStream_t s, int device) {
+  int sms = 148;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+  const size_t smem = sizeof(F32Smem);
+  const int64_t grid = ts.n_tiles < sms ? ts.n_tiles : sms;
+  if (grid <= 0) return cudaSuccess;
+  cudaError_t e;
+  if (in_kind == LAKE_IN_RAW) {
+    e = cudaFuncSetAttribute(mlp_fp32_kernel<LAKE_IN_RAW>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    mlp_fp32_kernel<LAKE_IN_RAW><<<(unsigned)grid, kF32Threads, smem, s>>>(in, ts, decisions,
+                                                                            logits);
+  } else {
+    e = cudaFuncSetAttribute(mlp_fp32_kernel<LAKE_IN_DIGITS>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    mlp_fp32_kernel<LAKE_IN_DIGITS><<<(unsigned)grid, kF32Threads, smem, s>>>(
+        in, ts, decisions, logits);
+  }
+  count_launch();
+  return cudaGetLastError();
+}
+
+}  // namespace lake

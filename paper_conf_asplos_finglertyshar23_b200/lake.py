@@ -1,0 +1,203 @@
+"""Thin Python binding of the C ABI in include/lake_linnos.h (argument marshalling only).
+
+Every function has the C name without the ``lake_linnos_`` prefix and the same argument
+order; device buffers are torch CUDA tensors (or raw integer pointers), streams default to
+torch's current stream. All arithmetic runs in liblake_linnos.so's CUDA kernels; there is
+no CPU fallback: if the library is missing or fails to load, every call raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "liblake_linnos.so")
+
+# enums / flags (mirrors include/lake_linnos.h)
+LAKE_OK, LAKE_ERR_INVAL, LAKE_ERR_NOMODEL, LAKE_ERR_CUDA, LAKE_ERR_NOMEM, LAKE_ERR_UNSUPPORTED = range(6)
+LAKE_ARCH_NN, LAKE_ARCH_NN1, LAKE_ARCH_NN2 = 0, 1, 2
+LAKE_IN_DIGITS, LAKE_IN_RAW = 0x00, 0x01
+LAKE_PREC_FP32, LAKE_PREC_F16, LAKE_PREC_BF16, LAKE_PREC_TF32, LAKE_PREC_AUTO = (
+    0x00, 0x10, 0x20, 0x30, 0x70)
+LAKE_MAX_MODELS = 1024
+LAKE_AUTO_TC_MIN_N = 2048
+
+PREC_FLAGS = {"fp32": LAKE_PREC_FP32, "f16": LAKE_PREC_F16, "bf16": LAKE_PREC_BF16,
+              "tf32": LAKE_PREC_TF32, "auto": LAKE_PREC_AUTO}
+
+# every symbol include/lake_linnos.h declares (checked by tests/test_abi.py)
+EXPORTS = (
+    "lake_linnos_blob_floats", "lake_linnos_load_weights", "lake_linnos_unload",
+    "lake_linnos_model_arch", "lake_linnos_digitize", "lake_linnos_infer",
+    "lake_linnos_workspace_bytes", "lake_linnos_infer_multi", "lake_linnos_multi_group",
+    "lake_linnos_multi_grouped", "lake_linnos_multi_status", "lake_linnos_host_staging_bytes",
+    "lake_linnos_infer_host", "lake_linnos_launch_count", "lake_linnos_reset_launch_count",
+    "lake_linnos_profile_enable", "lake_linnos_profile_read", "lake_linnos_strerror",
+)
+
+
+class LakeError(RuntimeError):
+    def __init__(self, status: int, what: str):
+        super().__init__(f"{what}: {strerror(status)} ({status})")
+        self.status = status
+
+
+_lib = None
+
+
+def lib():
+    """Load liblake_linnos.so (built in-tree by `make`). Raises if it is missing."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"{LIB_PATH} is missing: run `make` (or __graft_entry__.build())")
+        L = ctypes.CDLL(LIB_PATH)
+        P, I32, I64, U32, SZ = (ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64,
+                                ctypes.c_uint32, ctypes.c_size_t)
+        sig = {
+            "lake_linnos_blob_floats": (SZ, [I32]),
+            "lake_linnos_load_weights": (ctypes.c_int, [I32, I32, P, SZ, I32]),
+            "lake_linnos_unload": (ctypes.c_int, [I32, I32]),
+            "lake_linnos_model_arch": (ctypes.c_int, [I32, I32, P]),
+            "lake_linnos_digitize": (ctypes.c_int, [P, I64, P, P]),
+            "lake_linnos_infer": (ctypes.c_int, [P, U32, I64, I32, P, P, P]),
+            "lake_linnos_workspace_bytes": (SZ, [I64]),
+            "lake_linnos_infer_multi": (ctypes.c_int, [P, U32, I64, P, P, P, P, SZ, P]),
+            "lake_linnos_multi_group": (ctypes.c_int, [I64, P, P, SZ, P]),
+            "lake_linnos_multi_grouped": (ctypes.c_int, [P, U32, I64, P, P, P, SZ, P]),
+            "lake_linnos_multi_status": (ctypes.c_int, [P, SZ, P, P]),
+            "lake_linnos_host_staging_bytes": (SZ, [I64, U32]),
+            "lake_linnos_infer_host": (ctypes.c_int, [P, U32, I64, I32, P, P, P, P, SZ, P]),
+            "lake_linnos_launch_count": (ctypes.c_uint64, []),
+            "lake_linnos_reset_launch_count": (None, []),
+            "lake_linnos_profile_enable": (ctypes.c_int, [ctypes.c_int]),
+            "lake_linnos_profile_read": (ctypes.c_int, [P, P]),
+            "lake_linnos_strerror": (ctypes.c_char_p, [ctypes.c_int]),
+        }
+        for name, (res, args) in sig.items():
+            f = getattr(L, name)
+            f.restype = res
+            f.argtypes = args
+        _lib = L
+    return _lib
+
+
+def strerror(status: int) -> str:
+    return lib().lake_linnos_strerror(status).decode()
+
+
+def _ptr(x):
+    """Device/host pointer of a torch tensor, numpy array, int, or None."""
+    if x is None:
+        return None
+    if isinstance(x, int):
+        return x
+    if isinstance(x, np.ndarray):
+        return x.ctypes.data
+    return x.data_ptr()
+
+
+def _stream(stream):
+    if stream is None:
+        import torch
+        return torch.cuda.current_stream().cuda_stream
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+def _check(rc: int, what: str) -> None:
+    if rc != LAKE_OK:
+        raise LakeError(rc, what)
+
+
+def blob_floats(arch: int) -> int:
+    return int(lib().lake_linnos_blob_floats(arch))
+
+
+def load_weights(model_id: int, arch: int, blob: np.ndarray, device: int) -> None:
+    blob = np.ascontiguousarray(blob, dtype=np.float32)
+    _check(lib().lake_linnos_load_weights(model_id, arch, blob.ctypes.data, blob.size, device),
+           "load_weights")
+
+
+def unload(model_id: int, device: int) -> None:
+    _check(lib().lake_linnos_unload(model_id, device), "unload")
+
+
+def model_arch(model_id: int, device: int) -> int:
+    out = ctypes.c_int32(-1)
+    _check(lib().lake_linnos_model_arch(model_id, device, ctypes.byref(out)), "model_arch")
+    return out.value
+
+
+def digitize(raw, n: int, digits, stream=None) -> None:
+    _check(lib().lake_linnos_digitize(_ptr(raw), n, _ptr(digits), _stream(stream)), "digitize")
+
+
+def infer(inp, flags: int, n: int, model_id: int, decisions, logits=None, stream=None) -> None:
+    _check(lib().lake_linnos_infer(_ptr(inp), flags, n, model_id, _ptr(decisions), _ptr(logits),
+                                   _stream(stream)), "infer")
+
+
+def workspace_bytes(n: int) -> int:
+    return int(lib().lake_linnos_workspace_bytes(n))
+
+
+def infer_multi(inp, flags: int, n: int, model_ids, decisions, logits, workspace, ws_bytes: int,
+                stream=None) -> None:
+    _check(lib().lake_linnos_infer_multi(_ptr(inp), flags, n, _ptr(model_ids), _ptr(decisions),
+                                         _ptr(logits), _ptr(workspace), ws_bytes,
+                                         _stream(stream)), "infer_multi")
+
+
+def multi_group(n: int, model_ids, workspace, ws_bytes: int, stream=None) -> None:
+    _check(lib().lake_linnos_multi_group(n, _ptr(model_ids), _ptr(workspace), ws_bytes,
+                                         _stream(stream)), "multi_group")
+
+
+def multi_grouped(inp, flags: int, n: int, decisions, logits, workspace, ws_bytes: int,
+                  stream=None) -> None:
+    _check(lib().lake_linnos_multi_grouped(_ptr(inp), flags, n, _ptr(decisions), _ptr(logits),
+                                           _ptr(workspace), ws_bytes, _stream(stream)),
+           "multi_grouped")
+
+
+def multi_status(workspace, ws_bytes: int, stream=None) -> int:
+    out = ctypes.c_int64(0)
+    _check(lib().lake_linnos_multi_status(_ptr(workspace), ws_bytes, ctypes.addressof(out),
+                                          _stream(stream)), "multi_status")
+    return out.value
+
+
+def host_staging_bytes(n: int, flags: int) -> int:
+    return int(lib().lake_linnos_host_staging_bytes(n, flags))
+
+
+def infer_host(h_in, flags: int, n: int, model_id: int, h_model_ids, h_decisions, h_logits,
+               d_staging, staging_bytes: int, stream=None) -> None:
+    _check(lib().lake_linnos_infer_host(_ptr(h_in), flags, n, model_id, _ptr(h_model_ids),
+                                        _ptr(h_decisions), _ptr(h_logits), _ptr(d_staging),
+                                        staging_bytes, _stream(stream)), "infer_host")
+
+
+def launch_count() -> int:
+    return int(lib().lake_linnos_launch_count())
+
+
+def reset_launch_count() -> None:
+    lib().lake_linnos_reset_launch_count()
+
+
+def profile_enable(enable: bool) -> None:
+    _check(lib().lake_linnos_profile_enable(1 if enable else 0), "profile_enable")
+
+
+def profile_read():
+    ms = ctypes.c_double(0.0)
+    n = ctypes.c_int64(0)
+    _check(lib().lake_linnos_profile_read(ctypes.addressof(ms), ctypes.addressof(n)),
+           "profile_read")
+    return ms.value, n.value

@@ -1,0 +1,219 @@
+"""GPU parity: the CUDA path through the C ABI vs the oracle, element by element.
+
+Bars (BASELINE.json north_star):
+  digitisation            bit-exact (integer)
+  FP32 path               decisions AND logits bit-exact (reading R15 fixes the order)
+  tensor-core path fp16   logits within 2e-2 relative (S19 definition), decision agreement
+                          >= 99.9%, every disagreement with |logit0 - logit1| < 5e-2
+  tensor-core path bf16   reported; asserted against the looser bars stated in DESIGN.md §4
+Sizes span several tiles and a ragged tail (FP32 tile 64 rows, TC tile 256 rows).
+"""
+import numpy as np
+import pytest
+
+import oracle
+from gpu_util import cuda, run_infer, run_multi, tc_metrics
+from paper_conf_asplos_finglertyshar23_b200 import inputs, lake
+
+pytestmark = pytest.mark.gpu
+
+ARCHS = [0, 1, 2]
+RAGGED = [1, 63, 64, 65, 255, 257, 1000, 4096 + 17]
+
+
+@pytest.fixture(scope="module", autouse=True)
+def models():
+    import torch
+    torch.cuda.set_device(0)
+    for arch in ARCHS:
+        lake.load_weights(10 + arch, arch, inputs.weights(arch, 10 + arch), 0)
+    yield
+    for arch in ARCHS:
+        lake.unload(10 + arch, 0)
+
+
+def _trace(n, seed=77):
+    raw = inputs.device_trace("azure", max(n - n // 4, 1), seed, rerate=3.0)["raw"]
+    return np.ascontiguousarray(np.concatenate([raw, inputs.edge_raw(n - raw.shape[0], seed + 1)])[:n])
+
+
+# ------------------------------------------------------------------------- digitise
+@pytest.mark.parametrize("n", [1, 127, 129, 4095, 1 << 20])
+def test_digitize_bit_exact(n):
+    import torch
+    raw = inputs.edge_raw(n, seed=n)
+    d = torch.full((n, 32), 0xAB, dtype=torch.uint8, device="cuda:0")
+    lake.digitize(cuda(raw), n, d)
+    torch.cuda.synchronize()
+    got = d.cpu().numpy()
+    assert np.array_equal(got[:, :31], oracle.digitize(raw))
+    assert np.all(got[:, 31] == 0)
+
+
+def test_digitize_misaligned_output():
+    import torch
+    n = 1000
+    raw = inputs.edge_raw(n, seed=5)
+    buf = torch.zeros(n * 32 + 8, dtype=torch.uint8, device="cuda:0")
+    lake.digitize(cuda(raw), n, buf.data_ptr() + 4)
+    torch.cuda.synchronize()
+    got = buf.cpu().numpy()[4:4 + n * 32].reshape(n, 32)
+    assert np.array_equal(got[:, :31], oracle.digitize(raw))
+
+
+# ------------------------------------------------------------------------- FP32 path
+@pytest.mark.parametrize("arch", ARCHS)
+@pytest.mark.parametrize("n", RAGGED)
+def test_fp32_raw_bit_exact(arch, n):
+    raw = _trace(n)
+    lg, dec = run_infer(10 + arch, raw, lake.LAKE_IN_RAW | lake.LAKE_PREC_FP32)
+    rlg, rdec = oracle.infer_raw(arch, inputs.weights(arch, 10 + arch), raw, nthreads=0)
+    assert np.array_equal(dec, rdec)
+    assert np.array_equal(lg.view(np.uint32), rlg.view(np.uint32))
+
+
+@pytest.mark.parametrize("arch", ARCHS)
+def test_fp32_digits_input_bit_exact(arch):
+    n = 3000
+    raw = _trace(n, seed=91)
+    dig = np.zeros((n, 32), np.uint8)
+    dig[:, :31] = oracle.digitize(raw)
+    lg, dec = run_infer(10 + arch, dig, lake.LAKE_IN_DIGITS | lake.LAKE_PREC_FP32)
+    rlg, rdec = oracle.infer_digits(arch, inputs.weights(arch, 10 + arch), dig, nthreads=0)
+    assert np.array_equal(dec, rdec)
+    assert np.array_equal(lg.view(np.uint32), rlg.view(np.uint32))
+
+
+def test_fp32_without_logits():
+    raw = _trace(500)
+    _, dec = run_infer(12, raw, lake.LAKE_IN_RAW, logits=False)
+    _, rdec = oracle.infer_raw(2, inputs.weights(2, 12), raw, nthreads=0)
+    assert np.array_equal(dec, rdec)
+
+
+# ------------------------------------------------------------------------- tensor cores
+@pytest.mark.parametrize("arch", ARCHS)
+@pytest.mark.parametrize("n", [1, 255, 256, 257, 20000])
+def test_tc_f16_tolerance(arch, n):
+    raw = _trace(n, seed=5 + n)
+    lg, dec = run_infer(10 + arch, raw, lake.LAKE_IN_RAW | lake.LAKE_PREC_F16)
+    rlg, rdec = oracle.infer_raw(arch, inputs.weights(arch, 10 + arch), raw, nthreads=0)
+    m = tc_metrics(lg, dec, rlg, rdec)
+    assert m["max_rel"] <= 2e-2, m
+    assert m["max_disagree_margin"] < 5e-2, m
+    if n >= 20000:
+        assert m["agreement"] >= 0.999, m
+
+
+@pytest.mark.parametrize("arch", ARCHS)
+def test_tc_bf16_tolerance(arch):
+    n = 20000
+    raw = _trace(n, seed=33)
+    lg, dec = run_infer(10 + arch, raw, lake.LAKE_IN_RAW | lake.LAKE_PREC_BF16)
+    rlg, rdec = oracle.infer_raw(arch, inputs.weights(arch, 10 + arch), raw, nthreads=0)
+    m = tc_metrics(lg, dec, rlg, rdec)
+    print("bf16", arch, m)
+    # bf16 keeps 8 mantissa bits: DESIGN.md §4 states the looser bar it is held to
+    assert m["max_rel"] <= 8e-2, m
+    assert m["agreement"] >= 0.99, m
+    assert m["max_disagree_margin"] < 2e-1, m
+
+
+@pytest.mark.parametrize("arch", ARCHS)
+def test_tc_digits_equals_raw(arch):
+    n = 5000
+    raw = _trace(n, seed=3)
+    dig = np.zeros((n, 32), np.uint8)
+    dig[:, :31] = oracle.digitize(raw)
+    a = run_infer(10 + arch, raw, lake.LAKE_IN_RAW | lake.LAKE_PREC_F16)
+    b = run_infer(10 + arch, dig, lake.LAKE_IN_DIGITS | lake.LAKE_PREC_F16)
+    assert np.array_equal(a[0].view(np.uint32), b[0].view(np.uint32))
+    assert np.array_equal(a[1], b[1])
+
+
+@pytest.mark.parametrize("prec", [lake.LAKE_PREC_F16, lake.LAKE_PREC_FP32])
+def test_batch_independence(prec):
+    # results do not depend on batch composition (header: determinism)
+    raw = _trace(3000, seed=8)
+    full = run_infer(12, raw, lake.LAKE_IN_RAW | prec)
+    a = run_infer(12, raw[:1111], lake.LAKE_IN_RAW | prec)
+    b = run_infer(12, raw[1111:], lake.LAKE_IN_RAW | prec)
+    assert np.array_equal(full[0].view(np.uint32), np.concatenate([a[0], b[0]]).view(np.uint32))
+    assert np.array_equal(full[1], np.concatenate([a[1], b[1]]))
+
+
+# ------------------------------------------------------------------------- multi-model
+@pytest.fixture(scope="module")
+def multi_models():
+    import torch
+    torch.cuda.set_device(0)
+    ids = [100, 101, 102]
+    archs = [2, 0, 1]
+    for m, a in zip(ids, archs):
+        lake.load_weights(m, a, inputs.weights(a, m), 0)
+    yield dict(zip(ids, archs))
+    for m in ids:
+        lake.unload(m, 0)
+
+
+@pytest.mark.parametrize("prec", [lake.LAKE_PREC_FP32, lake.LAKE_PREC_F16])
+@pytest.mark.parametrize("split", [False, True])
+def test_multi_equals_per_model(multi_models, prec, split):
+    raw, mids = inputs.multi_device_trace(30000, 3, seed_base=400, rerate=3.0)
+    ids = np.array(list(multi_models))[mids]
+    lg, dec, unk = run_multi(raw, ids, lake.LAKE_IN_RAW | prec, split_calls=split)
+    assert unk == 0
+    for m in multi_models:
+        idx = np.nonzero(ids == m)[0]
+        slg, sdec = run_infer(m, raw[idx], lake.LAKE_IN_RAW | prec)
+        assert np.array_equal(dec[idx], sdec)
+        assert np.array_equal(lg[idx].view(np.uint32), slg.view(np.uint32))
+    if prec == lake.LAKE_PREC_FP32:
+        rlg, rdec = oracle.infer_multi_raw(
+            {m: (a, inputs.weights(a, m)) for m, a in multi_models.items()}, raw, ids, nthreads=0)
+        assert np.array_equal(dec, rdec)
+        assert np.array_equal(lg.view(np.uint32), rlg.view(np.uint32))
+
+
+def test_multi_unknown_ids(multi_models):
+    raw = _trace(4000, seed=12)
+    rng = np.random.default_rng(1)
+    ids = rng.choice(np.array([100, 101, 102, 7, -5, 5000], np.int64), size=4000).astype(np.int32)
+    lg, dec, unk = run_multi(raw, ids, lake.LAKE_IN_RAW | lake.LAKE_PREC_FP32)
+    bad = ~np.isin(ids, [100, 101, 102])
+    assert unk == int(bad.sum())
+    assert np.all(dec[bad] == 0) and np.all(np.isnan(lg[bad]))
+    rlg, rdec = oracle.infer_multi_raw(
+        {m: (a, inputs.weights(a, m)) for m, a in multi_models.items()}, raw, ids, nthreads=0)
+    assert np.array_equal(dec, rdec)
+
+
+def test_multi_order_invariance(multi_models):
+    raw, mids = inputs.multi_device_trace(9000, 3, seed_base=500, rerate=3.0)
+    ids = np.array(list(multi_models))[mids]
+    lg, dec, _ = run_multi(raw, ids, lake.LAKE_IN_RAW | lake.LAKE_PREC_F16)
+    p = np.random.default_rng(3).permutation(raw.shape[0])
+    lg2, dec2, _ = run_multi(raw[p], ids[p], lake.LAKE_IN_RAW | lake.LAKE_PREC_F16)
+    assert np.array_equal(dec[p], dec2)
+    assert np.array_equal(lg[p].view(np.uint32), lg2.view(np.uint32))
+
+
+# ------------------------------------------------------------------------- errors
+def test_error_codes_on_device():
+    import torch
+    x = torch.zeros((10, 9), dtype=torch.int32, device="cuda:0")
+    d = torch.zeros(10, dtype=torch.uint8, device="cuda:0")
+    with pytest.raises(lake.LakeError) as e:
+        lake.infer(x, lake.LAKE_IN_RAW, 10, 999, d)
+    assert e.value.status == lake.LAKE_ERR_NOMODEL
+    with pytest.raises(lake.LakeError) as e:
+        lake.infer(x, lake.LAKE_IN_RAW | lake.LAKE_PREC_TF32, 10, 12, d)
+    assert e.value.status == lake.LAKE_ERR_UNSUPPORTED
+    with pytest.raises(lake.LakeError) as e:
+        lake.infer(x.data_ptr() + 1, lake.LAKE_IN_RAW, 10, 12, d)
+    assert e.value.status == lake.LAKE_ERR_INVAL
+    lake.infer(x, lake.LAKE_IN_RAW, 0, 12, d)  # n == 0: no-op
+    with pytest.raises(lake.LakeError) as e:
+        lake.load_weights(5, 2, np.zeros(10, np.float32), 0)
+    assert e.value.status == lake.LAKE_ERR_INVAL
+    assert lake.model_arch(12, 0) == 2
