@@ -1,0 +1,487 @@
+#!/usr/bin/env python
+"""bench.py — batched LinnOS I/O-latency classification on B200 (LAKE's hot path).
+
+Metric (BASELINE.json): I/O inferences/s (and batch latency vs batch size, `--mode sweep`),
+1/2/4/8 B200, % of roofline. Default workload = BASELINE.json configs[4] ("C5"): 64 per-SSD
+NN+2 models, 2^24 interleaved I/Os, sharded across the ranks (strong scaling: the total is
+fixed). A step = one pass of the whole hot path over the rank's shard: model grouping
+(histogram / scan / scatter) + fused digitise -> 4 layers -> argmax on tcgen05 tensor cores
+(fp16 operands, fp32 accumulation), through the C ABI (lake_linnos_infer_multi).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C5] [--prec f16]
+    torchrun --nproc-per-node N bench.py --gpus N ...
+    python bench.py --impl reference ...     # the CPU oracle on the same workload
+    python bench.py --mode sweep             # C2 latency vs batch size (writes JSON lines)
+
+Inputs are synthetic and seeded (paper_conf_asplos_finglertyshar23_b200.inputs); weights
+are random init (no trained LinnOS weights are published). The oracle is executed only in
+the cpu_baseline leg and under --impl reference.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from paper_conf_asplos_finglertyshar23_b200 import inputs, shard  # noqa: E402
+
+ARCH_NAME = {0: "NN (31-256-2)", 1: "NN+1 (31-256-256-2)", 2: "NN+2 (31-256-256-256-2)"}
+# algorithmic FLOP per I/O, 2 per MAC, no padding
+ARCH_FLOPS = {0: 2 * (31 * 256 + 256 * 2), 1: 2 * (31 * 256 + 256 * 256 + 256 * 2),
+              2: 2 * (31 * 256 + 2 * 256 * 256 + 256 * 2)}
+RAW_BYTES = 36
+L2_BYTES = 126 * 1024 * 1024
+THROTTLE_BAD = ("hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown")
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=20)
+    p.add_argument("--warmup", type=int, default=5)
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--config", default="C5", choices=["C1", "C3", "C4", "C5"])
+    p.add_argument("--prec", default=None, choices=["fp32", "f16", "bf16"])
+    p.add_argument("--arch", type=int, default=None)
+    p.add_argument("--n", type=int, default=None)
+    p.add_argument("--mode", default="throughput", choices=["throughput", "sweep"])
+    p.add_argument("--sweep-out", default=None)
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-cpu", action="store_true")
+    p.add_argument("--cpu-seconds", type=float, default=12.0)
+    return p.parse_args()
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+# ------------------------------------------------------------------ distributed plumbing
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+def dist_init(world, local, backend="nccl"):
+    import torch
+    import torch.distributed as dist
+    if world > 1 and not dist.is_initialized():
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        if backend == "nccl":
+            torch.cuda.set_device(local)
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
+    return dist if world > 1 else None
+
+
+def max_over_ranks(x: float, dist, device=None) -> float:
+    if dist is None:
+        return x
+    import torch
+    t = torch.tensor([x], dtype=torch.float64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def barrier(dist):
+    if dist is not None:
+        dist.barrier()
+
+
+# ------------------------------------------------------------------ clocks (pynvml)
+class ClockSampler:
+    """Samples SM clock and throttle reasons every 50 ms during the timed region."""
+
+    REASONS = {
+        0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
+        0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
+        0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
+        0x100: "display_clock_setting",
+    }
+
+    def __init__(self, index: int):
+        self.ok = False
+        self.samples, self.reasons = [], 0
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception as e:  # pragma: no cover
+            log("clock sampler unavailable:", e)
+        self._stop = threading.Event()
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                self.reasons |= int(self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h))
+            except Exception:
+                pass
+            time.sleep(0.05)
+
+    def __enter__(self):
+        if self.ok:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        if self.ok:
+            self._stop.set()
+            self._t.join()
+
+    def summary(self):
+        if not self.ok or not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
+        names = [v for k, v in self.REASONS.items() if self.reasons & k and v != "gpu_idle"]
+        return {"sm_mhz": float(np.median(self.samples)), "sm_max_mhz": int(self.max_mhz),
+                "reasons": names, "samples": len(self.samples)}
+
+
+# ------------------------------------------------------------------ workload
+def workload(args, world, rank):
+    cfg = inputs.CONFIGS[args.config]
+    n = args.n or cfg["n"]
+    arch = cfg["arch"] if args.arch is None else args.arch
+    t = time.time()
+    w = inputs.workload(args.config, n=n, arch=arch)
+    log(f"[rank {rank}] generated {args.config} n={n} arch={arch} in {time.time() - t:.1f}s")
+    raw, ids = w["raw"], w["model_ids"]
+    n_models = cfg["models"]
+    p = shard.plan(ids, n_models, world)
+    if p["kind"] == "model_affine":
+        idx = shard.rank_indices(ids, p["owner"], rank)
+        mine = [m for m in range(n_models) if p["owner"][m] == rank]
+    else:
+        b, e = shard.range_split(n, world, rank)
+        idx = np.arange(b, e)
+        mine = list(range(n_models))
+    return dict(raw=np.ascontiguousarray(raw[idx]), ids=np.ascontiguousarray(ids[idx]),
+                models={m: w["models"][m] for m in mine}, n_total=n, arch=arch,
+                n_models=n_models, plan=p["kind"], imbalance=p["imbalance"],
+                full_raw=raw, full_ids=ids, all_models=w["models"])
+
+
+def config_obj(args, wl, prec, world, copies):
+    n = wl["n_total"]
+    return {
+        "workload": (f"{args.config}: {wl['n_models']} per-SSD {ARCH_NAME[wl['arch']].split()[0]} "
+                     f"model(s), {n} interleaved synthetic I/Os"
+                     + (", sharded across ranks (strong scaling)" if world > 1 else "")),
+        "n_ios": n, "models": wl["n_models"], "arch": ARCH_NAME[wl["arch"]],
+        "path": {"fp32": "CUDA-core FP32 (bit-exact)", "f16": "tcgen05 cta_group::2, fp16 in / fp32 acc",
+                 "bf16": "tcgen05 cta_group::2, bf16 in / fp32 acc"}[prec],
+        "input": "raw records (36 B/IO), digitised in-kernel; decisions out (1 B/IO)",
+        "api": "lake_linnos_infer_multi (group + fused MLP)",
+        "plan": wl["plan"], "imbalance": round(wl["imbalance"], 4),
+        "l2": (f"inputs larger than L2 ({copies} rotating input copies per rank, "
+               f">= 2x126 MB)" if copies > 1 else "inputs larger than L2"),
+    }
+
+
+# ------------------------------------------------------------------ CPU oracle timing
+def time_oracle(wl, seconds: float):
+    """The oracle, as it stands, on a bounded deterministic stride sample of the workload,
+    all host cores. Returns dict(value I/O-per-s, cores, sample)."""
+    import oracle
+    raw, ids, models = wl["full_raw"], wl["full_ids"], wl["all_models"]
+    cores = oracle.max_threads()
+    probe = np.arange(0, raw.shape[0], max(1, raw.shape[0] // 512))[:512]
+    t0 = time.perf_counter()
+    oracle.infer_multi_raw(models, raw[probe], ids[probe], nthreads=0)
+    per = (time.perf_counter() - t0) / probe.size
+    s = int(min(raw.shape[0], max(1024, seconds / max(per, 1e-9))))
+    stride = max(1, raw.shape[0] // s)
+    idx = np.arange(0, raw.shape[0], stride)[:s]
+    t0 = time.perf_counter()
+    oracle.infer_multi_raw(models, raw[idx], ids[idx], nthreads=0)
+    dt = time.perf_counter() - t0
+    return dict(value=idx.size / dt, unit="inferences/s", cores=cores, kind="oracle",
+                sample=(f"stride-{stride} sample of {idx.size} of the {raw.shape[0]} I/Os "
+                        f"({len(models)} models), {dt:.1f} s wall on {cores} threads"))
+
+
+# ------------------------------------------------------------------ our implementation
+def run_ours(args):
+    import torch
+    world, rank, local = dist_env()
+    if args.gpus != world and world > 1:
+        log(f"warning: --gpus {args.gpus} but WORLD_SIZE {world}")
+    dist = dist_init(world, local)
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    from paper_conf_asplos_finglertyshar23_b200 import lake
+
+    wl = workload(args, world, rank)
+    prec = args.prec or "f16"
+    flags = lake.LAKE_IN_RAW | lake.PREC_FLAGS[prec]
+    for m, (arch, blob) in wl["models"].items():
+        lake.load_weights(m, arch, blob, local)
+    n = wl["raw"].shape[0]
+    shard_bytes = n * RAW_BYTES
+    copies = max(1, math.ceil(2 * L2_BYTES / max(shard_bytes, 1))) if shard_bytes < 2 * L2_BYTES else 1
+    raw_np = wl["raw"].view(np.int32)
+    xs = [torch.from_numpy(raw_np).to(dev) for _ in range(copies)]
+    ids = torch.from_numpy(wl["ids"]).to(dev)
+    dec = torch.empty(max(n, 1), dtype=torch.uint8, device=dev)
+    wsb = lake.workspace_bytes(n)
+    ws = torch.empty(max(wsb, 1), dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream()
+
+    def step(i):
+        lake.infer_multi(xs[i % copies], flags, n, ids, dec, None, ws, wsb, stream)
+
+    for i in range(args.warmup):
+        step(i)
+    torch.cuda.synchronize()
+    barrier(dist)
+    torch.cuda.synchronize()
+    lake.reset_launch_count()
+    lake.profile_enable(True)
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        ev0.record(stream)
+        for i in range(args.steps):
+            step(i)
+        ev1.record(stream)
+        torch.cuda.synchronize()
+    barrier(dist)
+    torch.cuda.synchronize()
+    launches = lake.launch_count()
+    kern_ms, kern_n = lake.profile_read()
+    lake.profile_enable(False)
+    ms = ev0.elapsed_time(ev1)
+    ms_max = max_over_ranks(ms, dist, dev)
+    kern_avg = kern_ms / max(kern_n, 1)
+    kern_avg_max = max_over_ranks(kern_avg, dist, dev)
+    n_max = max_over_ranks(float(n), dist, dev)
+    value = wl["n_total"] * args.steps / (ms_max / 1e3)
+
+    # ---- roofline of the dominant kernel (fused MLP) -------------------------------------
+    peaks = {}
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            peaks = json.load(f)
+    except Exception:
+        pass
+    if prec == "fp32":
+        # FP32 CUDA-core peak derived from the guide's unit counts
+        sm_mhz = peaks.get("sm_max_mhz", 1965.0)
+        peak, src = 148 * 128 * 2 * sm_mhz * 1e6 / 1e12, "derived: 148 SM x 128 FFMA x 2 x max clock"
+        bound = "alu"
+    else:
+        peak = peaks.get("bf16_tflops")
+        src = "measured (MEASURED_PEAKS.json bf16 burst; fp16:bf16 nominal ratio 1:1)"
+        if peak is None:
+            peak, src = 1590.0, "fallback (B200_PROFILING.md)"
+        bound = "tensor"
+    flops_launch = ARCH_FLOPS[wl["arch"]] * n_max
+    achieved = flops_launch / (kern_avg_max / 1e3) / 1e12
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tpath):
+        try:
+            with open(tpath) as f:
+                tj = json.load(f)
+            key = f"{args.config}_{prec}_g{world}"
+            traffic = tj.get(key)
+        except Exception:
+            traffic = None
+    roofline = {"bound": bound, "achieved": round(achieved, 2), "peak": round(peak, 1),
+                "unit": "TFLOP/s", "frac": round(achieved / peak, 4), "traffic": traffic,
+                "kernel": "mlp_tc_kernel" if prec != "fp32" else "mlp_fp32_kernel",
+                "kernel_ms": round(kern_avg_max, 4), "flops_per_launch": flops_launch,
+                "peak_source": src,
+                "kernel_share_of_step": round(kern_avg_max / (ms_max / args.steps), 4)}
+
+    # ---- end to end through the C ABI with host buffers ----------------------------------
+    e2e = None
+    if not args.no_e2e:
+        h_in = torch.from_numpy(raw_np).pin_memory()
+        h_ids = torch.from_numpy(wl["ids"]).pin_memory()
+        h_dec = torch.empty(max(n, 1), dtype=torch.uint8).pin_memory()
+        stb = lake.host_staging_bytes(n, flags)
+        stg = torch.empty(max(stb, 1), dtype=torch.uint8, device=dev)
+        e_steps = max(1, min(args.steps, 5))
+        lake.infer_host(h_in, flags, n, -1, h_ids, h_dec, None, stg, stb, stream)
+        barrier(dist)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for _ in range(e_steps):
+            lake.infer_host(h_in, flags, n, -1, h_ids, h_dec, None, stg, stb, stream)
+        e_ms = (time.perf_counter() - t0) * 1e3 / e_steps
+        e_ms = max_over_ranks(e_ms, dist, dev)
+        e2e = {"value": round(wl["n_total"] / (e_ms / 1e3), 1), "unit": "inferences/s",
+               "h2d_bytes_per_step": int(n * (RAW_BYTES + 4)), "d2h_bytes_per_step": int(n),
+               "ms_per_step": round(e_ms, 3),
+               "how": "lake_linnos_infer_host: pinned H2D of raw+ids, group+fused MLP, D2H "
+                      "of decisions, stream sync; host wall clock, max over ranks"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cpu = time_oracle(wl, args.cpu_seconds)
+        cpu["value"] = round(cpu["value"], 1)
+
+    if rank == 0:
+        line = {
+            "metric": "I/O inferences/sec", "value": round(value, 1), "unit": "inferences/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(ms_max / args.steps, 4), "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": prec,
+            "data": "synthetic (seeded traces shaped like PAPER.md Table 4; random-init weights)",
+            "config": config_obj(args, wl, prec, world, copies),
+            "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+            "gpu_launches": int(launches), "clocks": clk.summary(),
+        }
+        print(json.dumps(line), flush=True)
+    if dist is not None:
+        dist.destroy_process_group()
+
+
+# ------------------------------------------------------------------ reference arm (oracle)
+def run_reference(args):
+    world, rank, _ = dist_env()
+    if rank != 0:
+        return
+    import oracle
+    cfg = inputs.CONFIGS[args.config]
+    n = args.n or cfg["n"]
+    arch = cfg["arch"] if args.arch is None else args.arch
+    w = inputs.workload(args.config, n=n, arch=arch)
+    raw, ids, models = w["raw"], w["model_ids"], w["models"]
+    cores = oracle.max_threads()
+    # per-step sample sized for ~3 s of oracle work so the whole run takes a few minutes
+    probe = np.arange(0, n, max(1, n // 256))[:256]
+    t0 = time.perf_counter()
+    oracle.infer_multi_raw(models, raw[probe], ids[probe], nthreads=0)
+    per = (time.perf_counter() - t0) / probe.size
+    s = int(min(n, max(256, 3.0 / max(per, 1e-9))))
+    stride = max(1, n // s)
+    idx = np.arange(0, n, stride)[:s]
+    r, i_ = raw[idx], ids[idx]
+    for _ in range(args.warmup):
+        oracle.infer_multi_raw(models, r, i_, nthreads=0)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        oracle.infer_multi_raw(models, r, i_, nthreads=0)
+    dt = time.perf_counter() - t0
+    value = idx.size * args.steps / dt
+    sample = (f"each step: stride-{stride} sample of {idx.size} of the {n} I/Os of "
+              f"{args.config} ({len(models)} models), oracle on {cores} host threads")
+    line = {
+        "impl": "reference", "metric": "I/O inferences/sec", "value": round(value, 1),
+        "unit": "inferences/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(dt * 1e3 / args.steps, 3), "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "fp32",
+        "data": "synthetic (seeded traces shaped like PAPER.md Table 4; random-init weights)",
+        "config": {"workload": f"{args.config}: {len(models)} per-SSD "
+                               f"{ARCH_NAME[arch].split()[0]} model(s), {n} I/Os (sampled per step)",
+                   "n_ios": n, "models": len(models), "arch": ARCH_NAME[arch]},
+        "cpu_baseline": {"value": round(value, 1), "unit": "inferences/s", "cores": cores,
+                         "kind": "oracle", "sample": sample},
+        "e2e": {"value": round(value, 1), "unit": "inferences/s", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------ C2: latency sweep
+def run_sweep(args):
+    """Batch latency vs batch size (BASELINE configs[1], Fig. 8): end-to-end
+    (pinned H2D -> infer -> D2H -> sync, host clock) and device-only, per arch x path, and
+    the 1-thread oracle for the same batch; crossover = smallest b where GPU e2e < CPU."""
+    import torch
+    import oracle
+    from paper_conf_asplos_finglertyshar23_b200 import lake
+    torch.cuda.set_device(0)
+    dev = torch.device("cuda", 0)
+    stream = torch.cuda.current_stream()
+    sizes = [1 << k for k in range(13)]
+    raw_all = inputs.device_trace("azure", max(sizes), 1200, 1.0)["raw"]
+    out = []
+    for arch in (0, 1, 2):
+        blob = inputs.weights(arch, 0)
+        lake.load_weights(40 + arch, arch, blob, 0)
+        for prec in ("fp32", "f16", "bf16"):
+            flags = lake.LAKE_IN_RAW | lake.PREC_FLAGS[prec]
+            cross = None
+            for b in sizes:
+                raw = np.ascontiguousarray(raw_all[:b])
+                h_in = torch.from_numpy(raw.view(np.int32)).pin_memory()
+                h_dec = torch.empty(b, dtype=torch.uint8).pin_memory()
+                d_in = torch.empty((b, 9), dtype=torch.int32, device=dev)
+                d_dec = torch.empty(b, dtype=torch.uint8, device=dev)
+                reps, warm = 200, 20
+
+                def once():
+                    d_in.copy_(h_in, non_blocking=True)
+                    lake.infer(d_in, flags, b, 40 + arch, d_dec, None, stream)
+                    h_dec.copy_(d_dec, non_blocking=True)
+                    stream.synchronize()
+                for _ in range(warm):
+                    once()
+                ts = []
+                for _ in range(reps):
+                    t0 = time.perf_counter()
+                    once()
+                    ts.append((time.perf_counter() - t0) * 1e6)
+                ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                ev0.record(stream)
+                for _ in range(reps):
+                    lake.infer(d_in, flags, b, 40 + arch, d_dec, None, stream)
+                ev1.record(stream)
+                torch.cuda.synchronize()
+                dev_us = ev0.elapsed_time(ev1) * 1e3 / reps
+                # 1-thread oracle for the same batch
+                oreps = max(1, min(50, int(2e4 / (b * (1 + 15 * arch)))))
+                t0 = time.perf_counter()
+                for _ in range(oreps):
+                    oracle.infer_raw(arch, blob, raw, nthreads=1)
+                cpu_us = (time.perf_counter() - t0) * 1e6 / oreps
+                med = float(np.median(ts))
+                if cross is None and med < cpu_us:
+                    cross = b
+                row = dict(arch=ARCH_NAME[arch], prec=prec, batch=b, e2e_us_median=round(med, 2),
+                           e2e_us_p99=round(float(np.percentile(ts, 99)), 2),
+                           device_us=round(dev_us, 2), cpu_1thread_us=round(cpu_us, 2))
+                out.append(row)
+                log(json.dumps(row))
+            out.append(dict(arch=ARCH_NAME[arch], prec=prec, crossover_batch=cross))
+            log(json.dumps(out[-1]))
+        lake.unload(40 + arch, 0)
+    path = args.sweep_out or os.path.join(ROOT, "gpurun_out", "sweep.jsonl")
+    os.makedirs(os.path.dirname(path), exist_ok=True)
+    with open(path, "w") as f:
+        for r in out:
+            f.write(json.dumps(r) + "\n")
+    print(json.dumps({"metric": "batch latency vs batch size (C2)", "rows": len(out),
+                      "crossovers": [r for r in out if "crossover_batch" in r]}))
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+    elif args.mode == "sweep":
+        run_sweep(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -158,10 +158,6 @@ void build_tc_image(const BlobView &v, uint8_t *img /* 2 * bytes */, size_t byte
       const int o = rank * (kTcOutN / 2) + n;
       for (int k = 0; k < 256; ++k) put(wo + umma_off(n, k, kTcOutN / 2), o < 2 ? v.W[nh][o * 256 + k] : 0.0f);
     }
-    float *bias = reinterpret_cast<float *>(base + wo + kTcWoHalfBytes);
-    for (int l = 0; l < nh; ++l) std::memcpy(bias + l * 256, v.b[l], 256 * 4);
-    bias[nh * 256 + 0] = v.b[nh][0];
-    bias[nh * 256 + 1] = v.b[nh][1];
   }
 }
 

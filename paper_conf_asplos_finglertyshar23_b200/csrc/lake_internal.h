@@ -33,9 +33,10 @@ constexpr int kTcOutN = 16;                                 // 2 classes padded 
 constexpr uint32_t kTcW0HalfBytes = 128 * kTcK0 * 2;        // 8 KB
 constexpr uint32_t kTcWhHalfBytes = 128 * kHidden * 2;      // 64 KB
 constexpr uint32_t kTcWoHalfBytes = (kTcOutN / 2) * kHidden * 2;  // 4 KB
-__host__ __device__ constexpr uint32_t tc_bias_floats(int nh) { return nh * kHidden + 4; }
+// Per-rank SMEM weight image: W0 half | hidden-layer halves | W_out half (biases stay in
+// global memory: the epilogue reads them through L1).
 __host__ __device__ constexpr uint32_t tc_image_bytes(int nh) {
-  return kTcW0HalfBytes + (nh - 1) * kTcWhHalfBytes + kTcWoHalfBytes + tc_bias_floats(nh) * 4;
+  return kTcW0HalfBytes + (nh - 1) * kTcWhHalfBytes + kTcWoHalfBytes;
 }
 
 struct DevModel {

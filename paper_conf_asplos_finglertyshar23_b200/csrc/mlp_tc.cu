@@ -55,7 +55,7 @@ __host__ __device__ constexpr Layout tc_layout(int nh_layout) {
 // barrier slots (8 bytes each) inside the barrier block
 enum : uint32_t {
   B_WLOAD = 0, B_WREADY = 1, B_XFULL = 2, B_XEMPTY = 4, B_DFULL = 6, B_HREADY = 8,
-  B_TILEDONE = 12, B_COUNT = 13
+  B_WFREE = 12, B_COUNT = 13
 };
 constexpr uint32_t kTmemSlot = B_COUNT * 8;  // u32 TMEM base address
 
@@ -83,7 +83,6 @@ __device__ __forceinline__ TileInfo tile_info(const TileSched &ts, int64_t t) {
 __device__ __forceinline__ uint32_t img_w0() { return 0; }
 __device__ __forceinline__ uint32_t img_wh(int l) { return kTcW0HalfBytes + (l - 1) * kTcWhHalfBytes; }
 __device__ __forceinline__ uint32_t img_wo(int nh) { return kTcW0HalfBytes + (nh - 1) * kTcWhHalfBytes; }
-__device__ __forceinline__ uint32_t img_bias(int nh) { return img_wo(nh) + kTcWoHalfBytes; }
 
 template <int PREC, int IN_KIND>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
@@ -111,7 +110,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       ptx::mbar_init(bar(B_DFULL + i), 1);       // tcgen05.commit (multicast)
     }
     for (int i = 0; i < 4; ++i) ptx::mbar_init(bar(B_HREADY + i), 16);  // 8 warps x 2 CTAs
-    ptx::mbar_init(bar(B_TILEDONE), 8);          // local epilogue warps
+    ptx::mbar_init(bar(B_WFREE), 1);             // tcgen05.commit (multicast): old weights free
     ptx::fence_mbar_init();
   }
   if (warp == 0) {
@@ -127,16 +126,18 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
     // ================= weight loader (both CTAs) =================
     if (lane == 0) {
       const DevModel *cur = nullptr;
-      int64_t done = 0;
-      uint32_t wl_phase = 0;
+      uint32_t wl_phase = 0, wf_phase = 0;
       const uint32_t wready_leader = ptx::mapa(bar(B_WREADY), 0);
       for (int64_t t = t_begin; t < t_end; ++t) {
         const TileInfo ti = tile_info(ts, t);
         if (ti.model == cur || (cur && ti.model->tc_img[PREC] == cur->tc_img[PREC])) continue;
-        // the previous model's last tile must be fully finished in this CTA
-        while (done < t - t_begin) {
-          ptx::mbar_wait(bar(B_TILEDONE), (uint32_t)(done & 1));
-          ++done;
+        // Model switch: every MMA that reads the old weights must have completed. The MMA
+        // thread commits B_WFREE once per switch, after the old model's last MMA; it cannot
+        // commit the next one before this loader has signalled B_WREADY, so the two sides
+        // stay within one phase of each other.
+        if (cur) {
+          ptx::mbar_wait(bar(B_WFREE), wf_phase);
+          wf_phase ^= 1;
         }
         const uint32_t bytes = ti.model->tc_img_bytes;
         const uint8_t *src = ti.model->tc_img[PREC] + (size_t)rank * bytes;
@@ -208,6 +209,11 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           ptx::mma_commit_cg2(bar(B_DFULL + (g & 1)), 0x3);
           ++g;
         }
+        if (t + 1 < t_end) {
+          const DevModel *nm = tile_info(ts, t + 1).model;
+          if (!(nm == cur || nm->tc_img[PREC] == cur->tc_img[PREC]))
+            ptx::mma_commit_cg2(bar(B_WFREE), 0x3);  // old weights no longer read
+        }
       }
     }
   } else if (warp < 4) {
@@ -271,12 +277,10 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
     const uint32_t hh = (warp - 4) >> 2;   // which 32-column half of each 64-column chunk
     const uint32_t row = q * 32 + lane;    // row within this CTA's 128
     const uint32_t hready_leader0 = ptx::mapa(bar(B_HREADY), 0);
-    const float *img_f = reinterpret_cast<const float *>(smem);
     uint32_t g = 0, d_phase = 0;  // d_phase: bit b
     for (int64_t t = t_begin; t < t_end; ++t) {
       const TileInfo ti = tile_info(ts, t);
       const int nh = ti.model->nh;
-      const float *bias = img_f + img_bias(nh) / 4;
       for (int l = 0; l <= nh; ++l) {
         const uint32_t b = g & 1;
         ptx::mbar_wait(bar(B_DFULL + b), (d_phase >> b) & 1);
@@ -284,11 +288,17 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         ptx::tc_fence_after();
         const uint32_t tbase = tmem + ((q * 32) << 16) + b * 256;
         if (l < nh) {
-          const float *bl = bias + l * kHidden;
+          const float *bl = ti.model->b[l];  // fp32 biases in global memory (L1-resident)
           for (uint32_t kc = 0; kc < 4; ++kc) {
             const uint32_t col0 = kc * 64 + hh * 32;
             uint32_t r[32];
             ptx::tmem_ld_32x32b_x32(tbase + col0, r);
+            float bv[32];
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+              const float4 b4 = __ldg(reinterpret_cast<const float4 *>(bl + col0) + i);
+              bv[4 * i + 0] = b4.x; bv[4 * i + 1] = b4.y; bv[4 * i + 2] = b4.z; bv[4 * i + 3] = b4.w;
+            }
             ptx::tmem_ld_wait();
 #pragma unroll
             for (int gq = 0; gq < 4; ++gq) {
@@ -296,8 +306,8 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
 #pragma unroll
               for (int e = 0; e < 4; ++e) {
                 const int c = gq * 8 + e * 2;
-                const float v0 = __uint_as_float(r[c]) + bl[col0 + c];
-                const float v1 = __uint_as_float(r[c + 1]) + bl[col0 + c + 1];
+                const float v0 = __uint_as_float(r[c]) + bv[c];
+                const float v1 = __uint_as_float(r[c + 1]) + bv[c + 1];
                 p[e] = PREC == 0 ? ptx::relu_pack_f16(v0, v1) : ptx::relu_pack_bf16(v0, v1);
               }
               ptx::st_shared_v4(sbase + L.h + ((col0 >> 3) + gq) * kLboR128 + row * 16, p[0],
@@ -312,8 +322,8 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           uint32_t r[2];
           ptx::tmem_ld_32x32b_x2(tbase, r);
           ptx::tmem_ld_wait();
-          const float l0 = __uint_as_float(r[0]) + bias[nh * kHidden + 0];
-          const float l1 = __uint_as_float(r[1]) + bias[nh * kHidden + 1];
+          const float l0 = __uint_as_float(r[0]) + __ldg(ti.model->bout);
+          const float l1 = __uint_as_float(r[1]) + __ldg(ti.model->bout + 1);
           const int pos = (int)(rank * 128 + row);
           if (pos < ti.count) {
             const int64_t p = ti.begin + pos;
@@ -327,9 +337,6 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         }
         ++g;
       }
-      ptx::tc_fence_before();
-      __syncwarp();
-      if (lane == 0) ptx::mbar_arrive(bar(B_TILEDONE));
     }
   }
 

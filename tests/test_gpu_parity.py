@@ -217,3 +217,60 @@ def test_error_codes_on_device():
         lake.load_weights(5, 2, np.zeros(10, np.float32), 0)
     assert e.value.status == lake.LAKE_ERR_INVAL
     assert lake.model_arch(12, 0) == 2
+
+
+# ------------------------------------------------------------------------- full sizes
+@pytest.fixture(scope="module")
+def many_models():
+    import torch
+    torch.cuda.set_device(0)
+    spec = {200 + i: (i % 3) for i in range(6)}  # mixed archs -> mixed layer counts per tile
+    for m, a in spec.items():
+        lake.load_weights(m, a, inputs.weights(a, m), 0)
+    yield spec
+    for m in spec:
+        lake.unload(m, 0)
+
+
+@pytest.mark.parametrize("prec", [lake.LAKE_PREC_F16, lake.LAKE_PREC_FP32])
+def test_multi_many_tiles_and_switches(many_models, prec):
+    # ~2,300 tensor-core tiles over 74 CTA pairs: every pair runs many tiles and crosses
+    # model boundaries (weight reload protocol), at the launch configuration of the bench.
+    n = 600_000
+    raw, mids = inputs.multi_device_trace(n, 6, seed_base=900, rerate=3.0)
+    ids = np.array(list(many_models))[mids]
+    lg, dec, unk = run_multi(raw, ids, lake.LAKE_IN_RAW | prec)
+    assert unk == 0
+    rng = np.random.default_rng(0)
+    for m, a in many_models.items():
+        idx = np.nonzero(ids == m)[0]
+        slg, sdec = run_infer(m, raw[idx], lake.LAKE_IN_RAW | prec)
+        assert np.array_equal(dec[idx], sdec)
+        assert np.array_equal(lg[idx].view(np.uint32), slg.view(np.uint32))
+        smp = np.sort(rng.choice(idx, size=min(2000, idx.size), replace=False))
+        rlg, rdec = oracle.infer_raw(a, inputs.weights(a, m), raw[smp], nthreads=0)
+        if prec == lake.LAKE_PREC_FP32:
+            assert np.array_equal(dec[smp], rdec)
+            assert np.array_equal(lg[smp].view(np.uint32), rlg.view(np.uint32))
+        else:
+            met = tc_metrics(lg[smp], dec[smp], rlg, rdec)
+            assert met["max_rel"] <= 2e-2 and met["max_disagree_margin"] < 5e-2, met
+
+
+@pytest.mark.parametrize("prec", [lake.LAKE_PREC_F16, lake.LAKE_PREC_FP32])
+def test_c3_full_size_sampled(prec):
+    # BASELINE configs[2]: NN+2, 2^20 I/Os, in the launch configuration the bench uses;
+    # the oracle checks a 4,096-row sample (plus the ragged tail rows).
+    n = 1 << 20
+    raw = inputs.workload("C3", n=n)["raw"]
+    lg, dec = run_infer(12, raw, lake.LAKE_IN_RAW | prec)
+    rng = np.random.default_rng(1)
+    smp = np.unique(np.concatenate([rng.choice(n, 4096, replace=False), np.arange(n - 300, n)]))
+    rlg, rdec = oracle.infer_raw(2, inputs.weights(2, 12), raw[smp], nthreads=0)
+    if prec == lake.LAKE_PREC_FP32:
+        assert np.array_equal(dec[smp], rdec)
+        assert np.array_equal(lg[smp].view(np.uint32), rlg.view(np.uint32))
+    else:
+        met = tc_metrics(lg[smp], dec[smp], rlg, rdec)
+        assert met["max_rel"] <= 2e-2 and met["max_disagree_margin"] < 5e-2, met
+        assert met["agreement"] >= 0.999, met
