@@ -153,11 +153,6 @@ void build_tc_image(const BlobView &v, uint8_t *img /* 2 * bytes */, size_t byte
         for (int k = 0; k < 256; ++k)
           put(o + umma_off(n, k, 128), v.W[l][(size_t)(rank * 128 + n) * 256 + k]);
     }
-    const size_t wo = kTcW0HalfBytes + (size_t)(nh - 1) * kTcWhHalfBytes;
-    for (int n = 0; n < kTcOutN / 2; ++n) {
-      const int o = rank * (kTcOutN / 2) + n;
-      for (int k = 0; k < 256; ++k) put(wo + umma_off(n, k, kTcOutN / 2), o < 2 ? v.W[nh][o * 256 + k] : 0.0f);
-    }
   }
 }
 

@@ -29,14 +29,13 @@ constexpr int kF32ActStride = 68;   // floats per activation row in SMEM (64 + 4
 constexpr int kTcRowsPerCta = 128;
 constexpr int kTcTileRows = 256;
 constexpr int kTcK0 = 32;                                   // 31 digits + zero pad
-constexpr int kTcOutN = 16;                                 // 2 classes padded to N=16
 constexpr uint32_t kTcW0HalfBytes = 128 * kTcK0 * 2;        // 8 KB
 constexpr uint32_t kTcWhHalfBytes = 128 * kHidden * 2;      // 64 KB
-constexpr uint32_t kTcWoHalfBytes = (kTcOutN / 2) * kHidden * 2;  // 4 KB
-// Per-rank SMEM weight image: W0 half | hidden-layer halves | W_out half (biases stay in
-// global memory: the epilogue reads them through L1).
+// Per-rank SMEM weight image: W0 half | hidden-layer halves. The biases and the 2-wide
+// output layer stay fp32 (the epilogue stages them from the FP32 image: b[0] .. b[nh-1],
+// W_out[2][256], b_out[2] are contiguous there).
 __host__ __device__ constexpr uint32_t tc_image_bytes(int nh) {
-  return kTcW0HalfBytes + (nh - 1) * kTcWhHalfBytes + kTcWoHalfBytes;
+  return kTcW0HalfBytes + (nh - 1) * kTcWhHalfBytes;
 }
 
 struct DevModel {

@@ -47,22 +47,24 @@ __device__ __forceinline__ void fence_mbar_init() {
 __device__ __forceinline__ void mbar_arrive(uint32_t bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(bar) : "memory");
 }
-// Arrive on a barrier given by a shared::cluster address (own or peer CTA), release at
-// cluster scope so this thread's prior writes are visible to the waiter.
+// Arrive on a barrier given by a shared::cluster address (own or peer CTA). Default
+// semantics (.release.cta): the only consumer of data published this way is the tensor core
+// (async proxy), made visible by fence.proxy.async before the arrive. A .cluster-scope
+// release here compiles to MEMBAR.ALL + ERRBAR on every arrive.
 __device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_bar) {
-  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];"
-               :: "r"(cluster_bar) : "memory");
+  asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" :: "r"(cluster_bar) : "memory");
 }
 __device__ __forceinline__ void mbar_arrive_expect_tx(uint32_t bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;"
                :: "r"(bar), "r"(bytes) : "memory");
 }
-// Block until the phase with parity `parity` has completed (acquire, cluster scope).
+// Block until the phase with parity `parity` has completed (default .acquire.cta; an
+// .acquire.cluster wait compiles to CCTL.IVALL, an L1 invalidation, on every wait).
 __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
   asm volatile(
       "{\n\t.reg .pred p;\n"
       "LAKE_WAIT_%=:\n\t"
-      "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%0], %1;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
       "@!p bra LAKE_WAIT_%=;\n\t}"
       :: "r"(bar), "r"(parity) : "memory");
 }
