@@ -32,3 +32,17 @@ clean:
 	rm -rf build $(LIB) $(ORACLE) $(TRACESIM)
 
 .PHONY: all clean
+
+# timeline-trace build (development only; not loaded by the product path)
+TRACE_LIB := build/trace/liblake_linnos_trace.so
+trace: $(TRACE_LIB)
+$(TRACE_LIB): $(SRCS) $(HDRS)
+	@mkdir -p build/trace
+	$(NVCC) $(NVFLAGS) -DLAKE_TRACE -shared -o $@ $(SRCS) -lcudart 2> build/trace/ptxas.log || (cat build/trace/ptxas.log; false)
+.PHONY: trace
+
+# A/B variants of the fused kernel (development): make variant VAR=name DEFS="-D..."
+variant:
+	@mkdir -p build/var/$(VAR)
+	$(NVCC) $(NVFLAGS) $(DEFS) -shared -o build/var/$(VAR)/liblake_linnos.so $(SRCS) -lcudart 2> build/var/$(VAR)/ptxas.log || (cat build/var/$(VAR)/ptxas.log; false)
+.PHONY: variant

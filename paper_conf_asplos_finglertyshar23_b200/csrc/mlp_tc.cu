@@ -17,9 +17,9 @@
 //    the MMA of layer l+1 runs into one, the epilogue drains layer l from the other. The
 //    epilogue writes H in 64-column chunks and signals each, so layer l+1's MMA starts on
 //    K-chunk 0 while later chunks are still being converted.
-//  * Warp roles (12 warps): w0 weight loader + TMEM allocator, w1 MMA issuer (leader CTA,
-//    one thread), w2-3 digitisers (raw records -> fp16 digits, double-buffered X),
-//    w4-11 epilogue (tcgen05.ld -> +bias -> ReLU -> fp16 -> st.shared -> mbarrier; the last
+//  * Warp roles (20 warps): w0-1 digitisers (raw records -> fp16 digits, double-buffered
+//    X), w2 weight loader + TMEM allocator, w19 MMA issuer (leader CTA, one thread),
+//    w3-18 epilogue, 4 per TMEM lane quadrant, 16 columns of each 64-column chunk each (tcgen05.ld -> +bias -> ReLU -> fp16 -> st.shared -> mbarrier; the last
 //    layer: -> W_out dot products -> logits / decision). Biases and W_out (fp32) are staged
 //    into SMEM by the epilogue warps themselves whenever the tile's model changes.
 //  * Operand layout: K-major, SWIZZLE_NONE core matrices (8 rows x 16 B), core (rg, kg) at
@@ -41,15 +41,44 @@
 #include "lake_internal.h"
 #include "lake_ptx.cuh"
 
+// ---- optional timeline trace (make trace): clock64 stamps from the leader CTA of cluster 0
+#ifdef LAKE_TRACE
+// per-stream event logs: stream 0 MMA thread, 1 epilogue warp 4, 2 epilogue warp 11,
+// 3 digitiser; thread-local write index (no atomics), 2 u64 per event, 64K events each
+__device__ unsigned long long *g_lake_trace = nullptr;
+#define LAKE_TRACE_CAP (1u << 16)
+#define LAKE_TEV(kind, tile, layer, chunk)                                                   \
+  do {                                                                                    \
+    if (g_lake_trace && cid == 0 && rank == 0 && tr_stream >= 0 && tr_i < LAKE_TRACE_CAP) { \
+      unsigned long long *p_ = g_lake_trace + 2ull * (tr_stream * LAKE_TRACE_CAP + tr_i++);  \
+      p_[0] = ((unsigned long long)(kind) << 56) | ((unsigned long long)(tile) << 24) |     \
+              ((unsigned long long)(layer) << 8) | (unsigned long long)(chunk);              \
+      p_[1] = clock64();                                                                  \
+    }                                                                                     \
+  } while (0)
+#else
+#define LAKE_TEV(kind, tile, layer, chunk) do {} while (0)
+#endif
+enum TraceKind { T_XFULL = 1, T_TEMPTY = 2, T_HREADY = 3, T_COMMIT = 4, T_DFULL = 5,
+                 T_CHUNK = 6, T_LAYER_END = 7, T_XEMPTY = 8, T_XARRIVE = 9, T_ISSUED = 10,
+                 T_LDWAIT = 11, T_STS = 12, T_FENCE = 13 };
+
 namespace lake {
 namespace {
 
-constexpr int kThreads = 384;
+#ifndef LAKE_EPI_PER_Q
+#define LAKE_EPI_PER_Q 2
+#endif
+constexpr uint32_t kEpiPerQ = LAKE_EPI_PER_Q;      // epilogue warps per TMEM lane quadrant
+constexpr uint32_t kEpiWarps = 4 * kEpiPerQ;       // 16
+constexpr uint32_t kEpiCols = 64 / kEpiPerQ;       // columns per warp per 64-column chunk
+constexpr int kThreads = 32 * (3 + kEpiWarps + 1);  // digitisers(2) + loader + epi + MMA
 constexpr uint32_t kHBytes = 128 * kHidden * 2;   // 64 KB
 constexpr uint32_t kXBytes = 128 * kTcK0 * 2;     // 8 KB
 constexpr uint32_t kLboR128 = 128 * 16;           // K-direction core stride, 128-row operand
 constexpr uint32_t kPrmFloats = kMaxHiddenLayers * kHidden + 2 * kHidden + 4;  // biases|Wout|bout
-constexpr uint32_t kRedBytes = 2 * 128 * 2 * 4;   // output-layer half sums, double-buffered
+constexpr uint32_t kPrm2Words = (kMaxHiddenLayers - 1) * kHidden / 2;  // packed bias pairs
+constexpr uint32_t kRedBytes = (kEpiPerQ - 1) * 128 * 2 * 4;  // output-layer partial sums
 
 __host__ __device__ constexpr uint32_t align1k(uint32_t x) { return (x + 1023u) & ~1023u; }
 
@@ -61,9 +90,9 @@ __host__ __device__ constexpr Layout tc_layout(int nh_layout) {
   L.h = align1k(tc_image_bytes(nh_layout));
   L.x = L.h + kHBytes;
   L.prm = L.x + 2 * kXBytes;
-  L.red = L.prm + kPrmFloats * 4;
+  L.red = L.prm + kPrmFloats * 4 + kPrm2Words * 4;
   L.bar = L.red + kRedBytes;
-  L.total = L.bar + 256;
+  L.total = L.bar + 128;
   return L;
 }
 
@@ -74,12 +103,17 @@ enum : uint32_t {
 };
 constexpr uint32_t kTmemSlot = B_COUNT * 8;  // u32 TMEM base address
 
+// Per-tile schedule entry. Each role loads tile t+1's entry at the top of tile t (the
+// global loads then overlap tile t's work instead of stalling the next iteration).
 struct TileInfo {
   const DevModel *model;
+  const uint8_t *img;  // this model's weight image for the precision in use
   int64_t begin;
   int count;
+  int nh;
 };
 
+template <int PREC>
 __device__ __forceinline__ TileInfo tile_info(const TileSched &ts, int64_t t) {
   TileInfo ti;
   if (ts.tile_model) {
@@ -92,46 +126,74 @@ __device__ __forceinline__ TileInfo tile_info(const TileSched &ts, int64_t t) {
     const int64_t rem = ts.n - ti.begin;
     ti.count = (int)(rem < kTcTileRows ? rem : kTcTileRows);
   }
+  ti.img = ti.model->tc_img[PREC];
+  ti.nh = ti.model->nh;
   return ti;
 }
 
-template <int PREC>
-__device__ __forceinline__ bool same_weights(const DevModel *a, const DevModel *b) {
-  return a == b || (a && b && a->tc_img[PREC] == b->tc_img[PREC]);
-}
+// Warp roles. The scheduler arbitrates highest-warp-id first, so the latency-critical MMA
+// issuer takes the top warp and the epilogue the next eight; the digitisers and the loader
+// (off the critical path) sit below.
+#ifndef LAKE_MMA_WARP_LOW
+constexpr uint32_t kWarpDig = 0;    // warps 0-1: digitisers (64 threads)
+constexpr uint32_t kWarpLoad = 2;   // weight loader + TMEM allocator
+constexpr uint32_t kWarpEpi = 3;    // epilogue warps (kEpiPerQ per TMEM quadrant)
+constexpr uint32_t kWarpMma = kWarpEpi + kEpiWarps;  // MMA issuer (leader CTA, one thread)
+#else
+constexpr uint32_t kWarpMma = 0;
+constexpr uint32_t kWarpDig = 1;
+constexpr uint32_t kWarpLoad = 3;
+constexpr uint32_t kWarpEpi = 4;
+#endif
 
 __device__ __forceinline__ uint32_t img_w0() { return 0; }
 __device__ __forceinline__ uint32_t img_wh(int l) { return kTcW0HalfBytes + (l - 1) * kTcWhHalfBytes; }
 
-// H chunk epilogue for one warp: 32 rows x 32 columns of fp32 accumulator (+bias, ReLU)
-// -> packed fp16/bf16 -> H (K-major core-matrix layout).
-template <int PREC>
-__device__ __forceinline__ void epi_to_h(const uint32_t (&r)[32], const float *bl, uint32_t col0,
-                                         uint32_t hrow_addr) {
+// H chunk epilogue for one warp: 32 rows x 32 columns of fp32 accumulator -> packed
+// fp16/bf16 pairs -> + bias, ReLU (one packed FMA per pair) -> H (K-major core layout).
+// bias2 holds the layer's biases as packed pairs in the operand type.
+template <int PREC, int W>
+__device__ __forceinline__ void epi_to_h(const uint32_t (&r)[W], const uint32_t *bias2,
+                                         uint32_t col0, uint32_t hrow_addr) {
+  const uint32_t one2 = PREC == 0 ? 0x3C003C00u : 0x3F803F80u;
 #pragma unroll
-  for (int gq = 0; gq < 4; ++gq) {
+  for (int gq = 0; gq < W / 8; ++gq) {
+    const uint4 bb = *reinterpret_cast<const uint4 *>(bias2 + (col0 >> 1) + gq * 4);
+    const uint32_t bv[4] = {bb.x, bb.y, bb.z, bb.w};
     uint32_t p[4];
 #pragma unroll
     for (int e = 0; e < 4; ++e) {
       const int c = gq * 8 + e * 2;
-      const float v0 = __uint_as_float(r[c]) + bl[col0 + c];
-      const float v1 = __uint_as_float(r[c + 1]) + bl[col0 + c + 1];
-      p[e] = PREC == 0 ? ptx::relu_pack_f16(v0, v1) : ptx::relu_pack_bf16(v0, v1);
+      const float v0 = __uint_as_float(r[c]), v1 = __uint_as_float(r[c + 1]);
+      if (PREC == 0)
+        p[e] = ptx::hfma2_relu_f16(ptx::pack_f16(v0, v1), one2, bv[e]);
+      else
+        p[e] = ptx::hfma2_relu_bf16(ptx::pack_bf16(v0, v1), one2, bv[e]);
     }
     ptx::st_shared_v4(hrow_addr + ((col0 >> 3) + gq) * kLboR128, p[0], p[1], p[2], p[3]);
   }
 }
 
-// Last hidden layer: ReLU(acc + b) in fp32, accumulated straight into the two logits.
-__device__ __forceinline__ void epi_to_logits(const uint32_t (&r)[32], const float *bl,
-                                              const float *wo, uint32_t col0, float &p0,
-                                              float &p1) {
+// Last hidden layer: ReLU(acc + b) in fp32, accumulated straight into the two logits
+// (two partial sums per logit to halve the dependent-FMA chain).
+template <int W>
+__device__ __forceinline__ void epi_to_logits(const uint32_t (&r)[W], const float *bl,
+                                              const float *wo, uint32_t col0, float (&p)[4]) {
 #pragma unroll
-  for (int c = 0; c < 32; ++c) {
-    float h = __uint_as_float(r[c]) + bl[col0 + c];
-    h = h > 0.0f ? h : 0.0f;
-    p0 = fmaf(h, wo[col0 + c], p0);
-    p1 = fmaf(h, wo[kHidden + col0 + c], p1);
+  for (int c4 = 0; c4 < W / 4; ++c4) {
+    const float4 b4 = *reinterpret_cast<const float4 *>(bl + col0 + c4 * 4);
+    const float4 w0 = *reinterpret_cast<const float4 *>(wo + col0 + c4 * 4);
+    const float4 w1 = *reinterpret_cast<const float4 *>(wo + kHidden + col0 + c4 * 4);
+    const float bb[4] = {b4.x, b4.y, b4.z, b4.w};
+    const float ww0[4] = {w0.x, w0.y, w0.z, w0.w};
+    const float ww1[4] = {w1.x, w1.y, w1.z, w1.w};
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      float h = __uint_as_float(r[c4 * 4 + e]) + bb[e];
+      h = h > 0.0f ? h : 0.0f;
+      p[(e & 1) * 2 + 0] = fmaf(h, ww0[e], p[(e & 1) * 2 + 0]);
+      p[(e & 1) * 2 + 1] = fmaf(h, ww1[e], p[(e & 1) * 2 + 1]);
+    }
   }
 }
 
@@ -148,6 +210,11 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
   const uint32_t rank = ptx::cluster_ctarank();
   const uint32_t cid = ptx::cluster_id_x(), ncl = ptx::num_clusters_x();
 
+#ifdef LAKE_TRACE
+  const int tr_stream = (warp == kWarpMma && lane == 0) ? 0 : (warp == kWarpEpi && lane == 0) ? 1
+                      : (warp == kWarpMma - 1 && lane == 0) ? 2 : (threadIdx.x == 0) ? 3 : -1;
+  uint32_t tr_i = 0;
+#endif
   const int64_t n_tiles = ts.n_tiles_dev ? (int64_t)*ts.n_tiles_dev : ts.n_tiles;
   const int64_t t_begin = n_tiles * cid / ncl;
   const int64_t t_end = n_tiles * (cid + 1) / ncl;
@@ -159,13 +226,13 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       ptx::mbar_init(bar(B_XFULL + i), 2);       // one arrive per CTA digitiser group
       ptx::mbar_init(bar(B_XEMPTY + i), 1);      // tcgen05.commit (multicast)
       ptx::mbar_init(bar(B_DFULL + i), 1);       // tcgen05.commit (multicast)
-      ptx::mbar_init(bar(B_TEMPTY + i), 16);     // 8 epilogue warps x 2 CTAs
+      ptx::mbar_init(bar(B_TEMPTY + i), 2 * kEpiWarps);  // every epilogue warp, both CTAs
     }
-    for (int i = 0; i < 4; ++i) ptx::mbar_init(bar(B_HREADY + i), 16);
+    for (int i = 0; i < 4; ++i) ptx::mbar_init(bar(B_HREADY + i), 2 * kEpiWarps);
     ptx::mbar_init(bar(B_WFREE), 1);             // tcgen05.commit (multicast)
     ptx::fence_mbar_init();
   }
-  if (warp == 0) {
+  if (warp == kWarpLoad) {
     ptx::tmem_alloc_cg2(sbase + L.bar + kTmemSlot, 512);
     ptx::tmem_relinquish_cg2();
   }
@@ -174,15 +241,15 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
   ptx::tc_fence_after();
   const uint32_t tmem = *reinterpret_cast<volatile uint32_t *>(smem + L.bar + kTmemSlot);
 
-  if (warp == 0) {
+  if (warp == kWarpLoad) {
     // ================= weight loader (both CTAs) =================
     if (lane == 0) {
-      const DevModel *cur = nullptr;
+      const uint8_t *cur = nullptr;
       uint32_t wl_phase = 0, wf_phase = 0;
       const uint32_t wready_leader = ptx::mapa(bar(B_WREADY), 0);
       for (int64_t t = t_begin; t < t_end; ++t) {
-        const TileInfo ti = tile_info(ts, t);
-        if (same_weights<PREC>(ti.model, cur)) continue;
+        const TileInfo ti = tile_info<PREC>(ts, t);
+        if (ti.img == cur) continue;
         // Model switch: every MMA reading the old weights must have completed. The MMA
         // thread commits B_WFREE once per switch, after the old model's last MMA; it cannot
         // commit the next one before this loader has signalled B_WREADY (lag <= 1 phase).
@@ -191,7 +258,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           wf_phase ^= 1;
         }
         const uint32_t bytes = ti.model->tc_img_bytes;
-        const uint8_t *src = ti.model->tc_img[PREC] + (size_t)rank * bytes;
+        const uint8_t *src = ti.img + (size_t)rank * bytes;
         ptx::mbar_arrive_expect_tx(bar(B_WLOAD), bytes);
         for (uint32_t off = 0; off < bytes; off += 32768) {
           const uint32_t len = (bytes - off) < 32768 ? (bytes - off) : 32768;
@@ -200,57 +267,80 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         ptx::mbar_wait(bar(B_WLOAD), wl_phase);
         wl_phase ^= 1;
         ptx::mbar_arrive_cluster(wready_leader);
-        cur = ti.model;
+        cur = ti.img;
       }
     }
-  } else if (warp == 1) {
+  } else if (warp == kWarpMma) {
     // ================= MMA issuer (leader CTA, one thread) =================
     if (rank == 0 && lane == 0) {
       const uint32_t idesc = ptx::umma_idesc_f16(PREC, 256, 256);
-      const DevModel *cur = nullptr;
+      // descriptors: advancing K by 16 elements = +2 core matrices = +2*LBO bytes, i.e.
+      // +(2*LBO)>>4 in the 14-bit start-address field (no carry: SMEM < 256 KB)
+      constexpr uint64_t kStep = (2 * kLboR128) >> 4;
+      const uint64_t xdesc0 = ptx::umma_desc(sbase + L.x, kLboR128, 128);
+      const uint64_t xdesc1 = ptx::umma_desc(sbase + L.x + kXBytes, kLboR128, 128);
+      const uint64_t w0desc = ptx::umma_desc(sbase + img_w0(), kLboR128, 128);
+      const uint64_t hdesc = ptx::umma_desc(sbase + L.h, kLboR128, 128);
+      uint64_t whdesc[kMaxHiddenLayers];
+      for (int l = 1; l < kMaxHiddenLayers; ++l)
+        whdesc[l] = ptx::umma_desc(sbase + img_wh(l), kLboR128, 128);
+      const uint8_t *cur = nullptr;
       uint32_t w_phase = 0, g = 0, h_phase = 0, t_phase = 0;  // h/t_phase: one bit per slot
-      uint32_t uses[2] = {0, 0};
+      uint32_t used = 0;  // bit b: accumulator b has been written before
       int64_t it = 0;
       auto acquire_buf = [&](uint32_t b) {  // accumulator b must be drained by the epilogues
-        if (uses[b]++ > 0) {
+        if (used & (1u << b)) {
           ptx::mbar_wait(bar(B_TEMPTY + b), (t_phase >> b) & 1);
           t_phase ^= (1u << b);
         }
+        used |= (1u << b);
       };
+      TileInfo nxt;
+      if (t_begin < t_end) nxt = tile_info<PREC>(ts, t_begin);
       for (int64_t t = t_begin; t < t_end; ++t, ++it) {
-        const TileInfo ti = tile_info(ts, t);
-        if (!same_weights<PREC>(ti.model, cur)) {
+#ifdef LAKE_NO_PREFETCH
+        const TileInfo ti = tile_info<PREC>(ts, t);
+        if (t + 1 < t_end) nxt = tile_info<PREC>(ts, t + 1);
+#else
+        const TileInfo ti = nxt;
+        if (t + 1 < t_end) nxt = tile_info<PREC>(ts, t + 1);
+#endif
+        if (ti.img != cur) {
           ptx::mbar_wait(bar(B_WREADY), w_phase);
           w_phase ^= 1;
-          cur = ti.model;
+          cur = ti.img;
         }
-        const int nh = ti.model->nh;
+        const int nh = ti.nh;
         const uint32_t xb = (uint32_t)(it & 1);
         {  // layer 0: D = X[128(x2) x 32] * W0^T
           const uint32_t b = g & 1;
           acquire_buf(b);
+          LAKE_TEV(T_TEMPTY, it, 0, 0);
           ptx::mbar_wait(bar(B_XFULL + xb), (uint32_t)((it >> 1) & 1));
+          LAKE_TEV(T_XFULL, it, 0, 0);
           ptx::tc_fence_after();
           const uint32_t d = tmem + b * 256;
-          const uint32_t xa = sbase + L.x + xb * kXBytes;
+          const uint64_t xd = xb ? xdesc1 : xdesc0;
 #pragma unroll
           for (uint32_t s = 0; s < kTcK0 / 16; ++s)
-            ptx::mma_f16_cg2(d, ptx::umma_desc(xa + s * 2 * kLboR128, kLboR128, 128),
-                             ptx::umma_desc(sbase + img_w0() + s * 2 * kLboR128, kLboR128, 128),
-                             idesc, s);
+            ptx::mma_f16_cg2(d, xd + s * kStep, w0desc + s * kStep, idesc, s);
           ptx::mma_commit_cg2(bar(B_XEMPTY + xb), 0x3);
           ptx::mma_commit_cg2(bar(B_DFULL + b), 0x3);
+          LAKE_TEV(T_COMMIT, it, 0, 0);
           ++g;
         }
         for (int l = 1; l < nh; ++l) {  // hidden layers 1..nh-1 (K = 256)
           const uint32_t b = g & 1;
           acquire_buf(b);
+          LAKE_TEV(T_TEMPTY, it, l, 0);
           ptx::tc_fence_after();
           const uint32_t d = tmem + b * 256;
           for (uint32_t kc = 0; kc < 4; ++kc) {
             ptx::mbar_wait(bar(B_HREADY + kc), (h_phase >> kc) & 1);
             h_phase ^= (1u << kc);
+            LAKE_TEV(T_HREADY, it, l, kc);
             ptx::tc_fence_after();
+#ifdef LAKE_INLINE_DESC
 #pragma unroll
             for (uint32_t s = 0; s < 4; ++s) {
               const uint32_t ks = kc * 4 + s;
@@ -258,23 +348,34 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
                                ptx::umma_desc(sbase + img_wh(l) + ks * 2 * kLboR128, kLboR128, 128),
                                idesc, ks);
             }
+#else
+            const uint64_t wd = l == 1 ? whdesc[1] : whdesc[2];
+#pragma unroll
+            for (uint32_t s = 0; s < 4; ++s) {
+              const uint32_t ks = kc * 4 + s;
+              ptx::mma_f16_cg2(d, hdesc + ks * kStep, wd + ks * kStep, idesc, ks);
+            }
+#endif
+            LAKE_TEV(T_ISSUED, it, l, kc);
           }
           ptx::mma_commit_cg2(bar(B_DFULL + b), 0x3);
+          LAKE_TEV(T_COMMIT, it, l, 0);
           ++g;
         }
-        if (t + 1 < t_end && !same_weights<PREC>(tile_info(ts, t + 1).model, cur))
+        if (t + 1 < t_end && nxt.img != cur)
           ptx::mma_commit_cg2(bar(B_WFREE), 0x3);  // old weights no longer read
       }
     }
-  } else if (warp < 4) {
+  } else if (warp >= kWarpDig && warp < kWarpDig + 2) {
     // ================= digitisers: raw -> X (fp16/bf16 digits), 2 rows per thread ========
-    const uint32_t d = threadIdx.x - 64;  // 0..63
+    const uint32_t d = threadIdx.x - kWarpDig * 32;  // 0..63
     const uint32_t xfull_leader0 = ptx::mapa(bar(B_XFULL), 0);
     int64_t it = 0;
     for (int64_t t = t_begin; t < t_end; ++t, ++it) {
-      const TileInfo ti = tile_info(ts, t);
+      const TileInfo ti = tile_info<PREC>(ts, t);
       const uint32_t xb = (uint32_t)(it & 1);
       ptx::mbar_wait(bar(B_XEMPTY + xb), (uint32_t)(((it >> 1) & 1) ^ 1));
+      LAKE_TEV(T_XEMPTY, it, 0, 0);
       const uint32_t xs = sbase + L.x + xb * kXBytes;
 #pragma unroll
       for (int half = 0; half < 2; ++half) {
@@ -320,31 +421,47 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       ptx::fence_proxy_async_smem();
       ptx::named_bar_sync(1, 64);
       if (d == 0) ptx::mbar_arrive_cluster(xfull_leader0 + xb * 8);
+      LAKE_TEV(T_XARRIVE, it, 0, 0);
     }
-  } else {
+  } else if (warp >= kWarpEpi && warp < kWarpEpi + kEpiWarps) {
     // ================= epilogue =================
-    const uint32_t et = threadIdx.x - 128;  // 0..255
-    const uint32_t q = warp & 3;            // TMEM lane quadrant this warp may access
-    const uint32_t hh = (warp - 4) >> 2;    // which 32-column half of each 64-column chunk
+    constexpr uint32_t NE = kEpiWarps * 32;           // epilogue threads
+    constexpr int W = kEpiCols;
+    const uint32_t et = threadIdx.x - kWarpEpi * 32;  // 0..NE-1
+    const uint32_t q = warp & 3;                      // TMEM lane quadrant this warp may access
+    const uint32_t hh = (warp - kWarpEpi) >> 2;       // which W-column slice of each chunk
     const uint32_t row = q * 32 + lane;     // row within this CTA's 128
     const uint32_t hready_leader0 = ptx::mapa(bar(B_HREADY), 0);
     const uint32_t tempty_leader0 = ptx::mapa(bar(B_TEMPTY), 0);
     const uint32_t hrow = sbase + L.h + row * 16;
     float *prm = reinterpret_cast<float *>(smem + L.prm);
+    uint32_t *prm2 = reinterpret_cast<uint32_t *>(smem + L.prm + kPrmFloats * 4);
     float *red = reinterpret_cast<float *>(smem + L.red);
     const DevModel *cur = nullptr;
     uint32_t g = 0, d_phase = 0;  // d_phase: bit b
     int64_t it = 0;
+    TileInfo nxt;
+    if (t_begin < t_end) nxt = tile_info<PREC>(ts, t_begin);
     for (int64_t t = t_begin; t < t_end; ++t, ++it) {
-      const TileInfo ti = tile_info(ts, t);
-      const int nh = ti.model->nh;
+#ifdef LAKE_NO_PREFETCH
+      const TileInfo ti = tile_info<PREC>(ts, t);
+#else
+      const TileInfo ti = nxt;
+      if (t + 1 < t_end) nxt = tile_info<PREC>(ts, t + 1);
+#endif
+      const int nh = ti.nh;
       if (ti.model != cur) {
         // stage this model's fp32 biases | W_out | b_out (contiguous in its FP32 image)
         const uint32_t nf4 = (nh * kHidden + 2 * kHidden + 4) / 4;
-        ptx::named_bar_sync(2, 256);
+        ptx::named_bar_sync(2, NE);
         const float4 *src = reinterpret_cast<const float4 *>(ti.model->b[0]);
-        for (uint32_t i = et; i < nf4; i += 256) reinterpret_cast<float4 *>(prm)[i] = __ldg(src + i);
-        ptx::named_bar_sync(2, 256);
+        for (uint32_t i = et; i < nf4; i += NE) reinterpret_cast<float4 *>(prm)[i] = __ldg(src + i);
+        // hidden-layer biases feeding an MMA, as packed operand-type pairs
+        for (uint32_t i = et; i < (uint32_t)(nh - 1) * kHidden / 2; i += NE) {
+          const float2 bf = __ldg(reinterpret_cast<const float2 *>(ti.model->b[0]) + i);
+          prm2[i] = PREC == 0 ? ptx::pack_f16(bf.x, bf.y) : ptx::pack_bf16(bf.x, bf.y);
+        }
+        ptx::named_bar_sync(2, NE);
         cur = ti.model;
       }
       const float *wo = prm + nh * kHidden;
@@ -352,52 +469,69 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         const uint32_t b = g & 1;
         ptx::mbar_wait(bar(B_DFULL + b), (d_phase >> b) & 1);
         d_phase ^= (1u << b);
+        LAKE_TEV(T_DFULL, it, l, warp);
         ptx::tc_fence_after();
-        const uint32_t tbase = tmem + ((q * 32) << 16) + b * 256 + hh * 32;
+        const uint32_t tbase = tmem + ((q * 32) << 16) + b * 256 + hh * W;
         const float *bl = prm + l * kHidden;
-        uint32_t ra[32], rb[32];
-        ptx::tmem_ld_32x32b_x32(tbase, ra);
+        uint32_t ra[W], rb[W];
+        ptx::tmem_ld_cols<W>(tbase, ra);
         ptx::tmem_ld_wait();
         if (l + 1 < nh) {
           // hidden layer feeding another MMA: 4 chunks of 64 columns, TMEM loads of the next
           // chunk in flight while the current one is converted and stored
 #pragma unroll
           for (uint32_t kc = 0; kc < 4; ++kc) {
-            const uint32_t col0 = kc * 64 + hh * 32;
+            const uint32_t col0 = kc * 64 + hh * W;
             if (kc + 1 < 4) {
-              if (kc & 1) ptx::tmem_ld_32x32b_x32(tbase + (kc + 1) * 64, ra);
-              else ptx::tmem_ld_32x32b_x32(tbase + (kc + 1) * 64, rb);
+              if (kc & 1) ptx::tmem_ld_cols<W>(tbase + (kc + 1) * 64, ra);
+              else ptx::tmem_ld_cols<W>(tbase + (kc + 1) * 64, rb);
             }
-            if (kc & 1) epi_to_h<PREC>(rb, bl, col0, hrow);
-            else epi_to_h<PREC>(ra, bl, col0, hrow);
+            if (kc & 1) epi_to_h<PREC, W>(rb, prm2 + l * kHidden / 2, col0, hrow);
+            else epi_to_h<PREC, W>(ra, prm2 + l * kHidden / 2, col0, hrow);
+            LAKE_TEV(T_STS, it, l, kc);
             ptx::fence_proxy_async_smem();
+            LAKE_TEV(T_FENCE, it, l, kc);
             __syncwarp();
             if (lane == 0) ptx::mbar_arrive_cluster(hready_leader0 + kc * 8);
+            LAKE_TEV(T_CHUNK, it, l, kc);
             if (kc + 1 < 4) ptx::tmem_ld_wait();
+            LAKE_TEV(T_LDWAIT, it, l, kc);
           }
         } else {
           // last hidden layer: fold the 2-neuron output layer (fp32, CUDA cores)
-          float p0 = 0.0f, p1 = 0.0f;
+          float p[4] = {0.0f, 0.0f, 0.0f, 0.0f};
 #pragma unroll
           for (uint32_t kc = 0; kc < 4; ++kc) {
-            const uint32_t col0 = kc * 64 + hh * 32;
+            const uint32_t col0 = kc * 64 + hh * W;
             if (kc + 1 < 4) {
-              if (kc & 1) ptx::tmem_ld_32x32b_x32(tbase + (kc + 1) * 64, ra);
-              else ptx::tmem_ld_32x32b_x32(tbase + (kc + 1) * 64, rb);
+              if (kc & 1) ptx::tmem_ld_cols<W>(tbase + (kc + 1) * 64, ra);
+              else ptx::tmem_ld_cols<W>(tbase + (kc + 1) * 64, rb);
             }
-            if (kc & 1) epi_to_logits(rb, bl, wo, col0, p0, p1);
-            else epi_to_logits(ra, bl, wo, col0, p0, p1);
+            if (kc & 1) epi_to_logits<W>(rb, bl, wo, col0, p);
+            else epi_to_logits<W>(ra, bl, wo, col0, p);
             if (kc + 1 < 4) ptx::tmem_ld_wait();
           }
-          float *rd = red + (it & 1) * 256 + row * 2;
-          if (hh == 1) {
+          float p0 = p[0] + p[2], p1 = p[1] + p[3];
+          // combine the kEpiPerQ warps of this quadrant (slices hh = 1.. write partials)
+          if (hh > 0) {
+            float *rd = red + ((hh - 1) * 128 + row) * 2;
             rd[0] = p0;
             rd[1] = p1;
           }
-          ptx::named_bar_sync(3 + q, 64);  // the two warps sharing this quadrant
+          ptx::named_bar_sync(3 + q, 32 * kEpiPerQ);
           if (hh == 0) {
-            const float l0 = p0 + rd[0] + wo[2 * kHidden + 0];
-            const float l1 = p1 + rd[1] + wo[2 * kHidden + 1];
+#pragma unroll
+            for (uint32_t j = 0; j + 1 < kEpiPerQ; ++j) {
+              p0 += red[(j * 128 + row) * 2 + 0];
+              p1 += red[(j * 128 + row) * 2 + 1];
+            }
+          }
+          // NN (one layer per tile): nothing else orders the next tile's partial writes
+          // after this read, so close the exchange explicitly
+          if (nh == 1) ptx::named_bar_sync(3 + q, 32 * kEpiPerQ);
+          if (hh == 0) {
+            const float l0 = p0 + wo[2 * kHidden + 0];
+            const float l1 = p1 + wo[2 * kHidden + 1];
             const int pos = (int)(rank * 128 + row);
             if (pos < ti.count) {
               const int64_t pp = ti.begin + pos;
@@ -414,6 +548,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         ptx::tc_fence_before();
         __syncwarp();
         if (lane == 0) ptx::mbar_arrive_cluster(tempty_leader0 + b * 8);
+        LAKE_TEV(T_LAYER_END, it, l, warp);
         ++g;
       }
     }
@@ -422,7 +557,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
   __syncwarp();  // reconverge role lanes before the .aligned cluster barrier
   ptx::tc_fence_before();
   ptx::cluster_sync();
-  if (warp == 0) {
+  if (warp == kWarpLoad) {
     ptx::tc_fence_after();
     ptx::tmem_dealloc_cg2(tmem, 512);
   }
@@ -449,6 +584,12 @@ cudaError_t launch_t(const void *in, const TileSched &ts, int nh_layout, uint8_t
 }  // namespace
 
 size_t tc_smem_bytes(int nh_layout) { return tc_layout(nh_layout).total; }
+
+#ifdef LAKE_TRACE
+extern "C" int lake_trace_set(void *dev_buf) {
+  return (int)cudaMemcpyToSymbol(g_lake_trace, &dev_buf, sizeof(void *));
+}
+#endif
 
 cudaError_t launch_mlp_tc(const void *in, int in_kind, int prec, const TileSched &ts, int nh,
                           uint8_t *decisions, float *logits, cudaStream_t s, int device) {

@@ -14,6 +14,8 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "liblake_linnos.so")
+# development only: scripts/trace_tc.py points this at the timeline-trace build
+LIB_PATH = os.environ.get("LAKE_LINNOS_LIB", LIB_PATH)
 
 # enums / flags (mirrors include/lake_linnos.h)
 LAKE_OK, LAKE_ERR_INVAL, LAKE_ERR_NOMODEL, LAKE_ERR_CUDA, LAKE_ERR_NOMEM, LAKE_ERR_UNSUPPORTED = range(6)
