@@ -71,7 +71,13 @@ namespace {
 #endif
 constexpr uint32_t kEpiPerQ = LAKE_EPI_PER_Q;      // epilogue warps per TMEM lane quadrant
 constexpr uint32_t kEpiWarps = 4 * kEpiPerQ;       // 16
-constexpr uint32_t kEpiCols = 64 / kEpiPerQ;       // columns per warp per 64-column chunk
+#ifndef LAKE_CHUNKS
+#define LAKE_CHUNKS 8
+#endif
+constexpr uint32_t kChunks = LAKE_CHUNKS;          // H column chunks per layer (MMA K-chunks)
+constexpr uint32_t kChunkCols = kHidden / kChunks;
+constexpr uint32_t kEpiCols = kChunkCols / kEpiPerQ;  // columns per warp per chunk
+constexpr uint32_t kKStepsPerChunk = kChunkCols / 16;
 constexpr int kThreads = 32 * (3 + kEpiWarps + 1);  // digitisers(2) + loader + epi + MMA
 constexpr uint32_t kHBytes = 128 * kHidden * 2;   // 64 KB
 constexpr uint32_t kXBytes = 128 * kTcK0 * 2;     // 8 KB
@@ -92,14 +98,14 @@ __host__ __device__ constexpr Layout tc_layout(int nh_layout) {
   L.prm = L.x + 2 * kXBytes;
   L.red = L.prm + kPrmFloats * 4 + kPrm2Words * 4;
   L.bar = L.red + kRedBytes;
-  L.total = L.bar + 128;
+  L.total = L.bar + 256;
   return L;
 }
 
 // barrier slots (8 bytes each) inside the barrier block
 enum : uint32_t {
   B_WLOAD = 0, B_WREADY = 1, B_XFULL = 2, B_XEMPTY = 4, B_DFULL = 6, B_TEMPTY = 8,
-  B_HREADY = 10, B_WFREE = 14, B_COUNT = 15
+  B_HREADY = 10, B_WFREE = 10 + kChunks, B_COUNT = 11 + kChunks
 };
 constexpr uint32_t kTmemSlot = B_COUNT * 8;  // u32 TMEM base address
 
@@ -228,7 +234,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       ptx::mbar_init(bar(B_DFULL + i), 1);       // tcgen05.commit (multicast)
       ptx::mbar_init(bar(B_TEMPTY + i), 2 * kEpiWarps);  // every epilogue warp, both CTAs
     }
-    for (int i = 0; i < 4; ++i) ptx::mbar_init(bar(B_HREADY + i), 2 * kEpiWarps);
+    for (uint32_t i = 0; i < kChunks; ++i) ptx::mbar_init(bar(B_HREADY + i), 2 * kEpiWarps);
     ptx::mbar_init(bar(B_WFREE), 1);             // tcgen05.commit (multicast)
     ptx::fence_mbar_init();
   }
@@ -335,15 +341,15 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           LAKE_TEV(T_TEMPTY, it, l, 0);
           ptx::tc_fence_after();
           const uint32_t d = tmem + b * 256;
-          for (uint32_t kc = 0; kc < 4; ++kc) {
+          for (uint32_t kc = 0; kc < kChunks; ++kc) {
             ptx::mbar_wait(bar(B_HREADY + kc), (h_phase >> kc) & 1);
             h_phase ^= (1u << kc);
             LAKE_TEV(T_HREADY, it, l, kc);
             ptx::tc_fence_after();
 #ifdef LAKE_INLINE_DESC
 #pragma unroll
-            for (uint32_t s = 0; s < 4; ++s) {
-              const uint32_t ks = kc * 4 + s;
+            for (uint32_t s = 0; s < kKStepsPerChunk; ++s) {
+              const uint32_t ks = kc * kKStepsPerChunk + s;
               ptx::mma_f16_cg2(d, ptx::umma_desc(sbase + L.h + ks * 2 * kLboR128, kLboR128, 128),
                                ptx::umma_desc(sbase + img_wh(l) + ks * 2 * kLboR128, kLboR128, 128),
                                idesc, ks);
@@ -351,8 +357,8 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
 #else
             const uint64_t wd = l == 1 ? whdesc[1] : whdesc[2];
 #pragma unroll
-            for (uint32_t s = 0; s < 4; ++s) {
-              const uint32_t ks = kc * 4 + s;
+            for (uint32_t s = 0; s < kKStepsPerChunk; ++s) {
+              const uint32_t ks = kc * kKStepsPerChunk + s;
               ptx::mma_f16_cg2(d, hdesc + ks * kStep, wd + ks * kStep, idesc, ks);
             }
 #endif
@@ -473,43 +479,61 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         ptx::tc_fence_after();
         const uint32_t tbase = tmem + ((q * 32) << 16) + b * 256 + hh * W;
         const float *bl = prm + l * kHidden;
-        uint32_t ra[W], rb[W];
+        constexpr bool kPrefetch = W <= 32;  // two W-register buffers
+        uint32_t ra[W], rb[W];  // rb unused (eliminated) without prefetch
+        (void)rb;
         ptx::tmem_ld_cols<W>(tbase, ra);
         ptx::tmem_ld_wait();
         if (l + 1 < nh) {
-          // hidden layer feeding another MMA: 4 chunks of 64 columns, TMEM loads of the next
-          // chunk in flight while the current one is converted and stored
+          // hidden layer feeding another MMA: kChunks chunks; with two register buffers the
+          // TMEM load of chunk kc+1 is in flight while chunk kc is converted and stored
 #pragma unroll
-          for (uint32_t kc = 0; kc < 4; ++kc) {
-            const uint32_t col0 = kc * 64 + hh * W;
-            if (kc + 1 < 4) {
-              if (kc & 1) ptx::tmem_ld_cols<W>(tbase + (kc + 1) * 64, ra);
-              else ptx::tmem_ld_cols<W>(tbase + (kc + 1) * 64, rb);
+          for (uint32_t kc = 0; kc < kChunks; ++kc) {
+            const uint32_t col0 = kc * kChunkCols + hh * W;
+            if constexpr (kPrefetch) {
+              if (kc + 1 < kChunks) {
+                if (kc & 1) ptx::tmem_ld_cols<W>(tbase + (kc + 1) * kChunkCols, ra);
+                else ptx::tmem_ld_cols<W>(tbase + (kc + 1) * kChunkCols, rb);
+              }
+              if (kc & 1) epi_to_h<PREC, W>(rb, prm2 + l * kHidden / 2, col0, hrow);
+              else epi_to_h<PREC, W>(ra, prm2 + l * kHidden / 2, col0, hrow);
+            } else {
+              if (kc > 0) {
+                ptx::tmem_ld_cols<W>(tbase + kc * kChunkCols, ra);
+                ptx::tmem_ld_wait();
+              }
+              epi_to_h<PREC, W>(ra, prm2 + l * kHidden / 2, col0, hrow);
             }
-            if (kc & 1) epi_to_h<PREC, W>(rb, prm2 + l * kHidden / 2, col0, hrow);
-            else epi_to_h<PREC, W>(ra, prm2 + l * kHidden / 2, col0, hrow);
             LAKE_TEV(T_STS, it, l, kc);
             ptx::fence_proxy_async_smem();
             LAKE_TEV(T_FENCE, it, l, kc);
             __syncwarp();
             if (lane == 0) ptx::mbar_arrive_cluster(hready_leader0 + kc * 8);
             LAKE_TEV(T_CHUNK, it, l, kc);
-            if (kc + 1 < 4) ptx::tmem_ld_wait();
+            if (kPrefetch && kc + 1 < kChunks) ptx::tmem_ld_wait();
             LAKE_TEV(T_LDWAIT, it, l, kc);
           }
         } else {
           // last hidden layer: fold the 2-neuron output layer (fp32, CUDA cores)
           float p[4] = {0.0f, 0.0f, 0.0f, 0.0f};
 #pragma unroll
-          for (uint32_t kc = 0; kc < 4; ++kc) {
-            const uint32_t col0 = kc * 64 + hh * W;
-            if (kc + 1 < 4) {
-              if (kc & 1) ptx::tmem_ld_cols<W>(tbase + (kc + 1) * 64, ra);
-              else ptx::tmem_ld_cols<W>(tbase + (kc + 1) * 64, rb);
+          for (uint32_t kc = 0; kc < kChunks; ++kc) {
+            const uint32_t col0 = kc * kChunkCols + hh * W;
+            if constexpr (kPrefetch) {
+              if (kc + 1 < kChunks) {
+                if (kc & 1) ptx::tmem_ld_cols<W>(tbase + (kc + 1) * kChunkCols, ra);
+                else ptx::tmem_ld_cols<W>(tbase + (kc + 1) * kChunkCols, rb);
+              }
+              if (kc & 1) epi_to_logits<W>(rb, bl, wo, col0, p);
+              else epi_to_logits<W>(ra, bl, wo, col0, p);
+              if (kc + 1 < kChunks) ptx::tmem_ld_wait();
+            } else {
+              if (kc > 0) {
+                ptx::tmem_ld_cols<W>(tbase + kc * kChunkCols, ra);
+                ptx::tmem_ld_wait();
+              }
+              epi_to_logits<W>(ra, bl, wo, col0, p);
             }
-            if (kc & 1) epi_to_logits<W>(rb, bl, wo, col0, p);
-            else epi_to_logits<W>(ra, bl, wo, col0, p);
-            if (kc + 1 < 4) ptx::tmem_ld_wait();
           }
           float p0 = p[0] + p[2], p1 = p[1] + p[3];
           // combine the kEpiPerQ warps of this quadrant (slices hh = 1.. write partials)
