@@ -171,11 +171,14 @@ int lake_linnos_multi_status(const void *workspace, size_t ws_bytes, int64_t *n_
                              void *stream);
 
 /* End-to-end call with HOST buffers (the latency path of Fig. 8, "including data copying
- * latencies"): copies h_in (pinned host recommended) to the device, runs
- * lake_linnos_infer_multi (model_ids == NULL -> lake_linnos_infer on model_id), copies
- * decisions (and logits if h_logits != NULL) back, in chunks pipelined on `stream` and an
- * internal second stream, then synchronises. d_staging: device buffer of at least
- * lake_linnos_host_staging_bytes(n, flags) bytes. */
+ * latencies"): h_in (pinned host memory recommended, else the copies are
+ * synchronous) is processed in chunks of up to 2^20 I/Os through a 3-stage pipeline:
+ * host->device copy on an internal stream, lake_linnos_infer_multi (h_model_ids != NULL) or
+ * lake_linnos_infer(model_id) on `stream`, device->host copy of decisions (and logits if
+ * h_logits != NULL) on a second internal stream, so chunk i+1's upload and chunk i-1's
+ * download overlap chunk i's kernels. Synchronous: returns when every output is on the host.
+ * d_staging: device buffer of at least lake_linnos_host_staging_bytes(n, flags) bytes (two
+ * chunk slots). LAKE_PREC_AUTO is resolved once for the whole batch. */
 size_t lake_linnos_host_staging_bytes(int64_t n, uint32_t flags);
 int lake_linnos_infer_host(const void *h_in, uint32_t flags, int64_t n, int32_t model_id,
                            const int32_t *h_model_ids, uint8_t *h_decisions, float *h_logits,

@@ -506,12 +506,66 @@ int lake_linnos_multi_status(const void *workspace, size_t ws_bytes, int64_t *n_
   return cuda_status(e);
 }
 
+}  // extern "C"
+
+// ---- host-buffer path: chunked 3-stream pipeline ------------------------------------------
+// chunk i: H2D (copy stream) -> group + fused kernel (caller's stream) -> D2H (copy-back
+// stream), two staging slots, so the PCIe transfers of neighbouring chunks overlap compute.
+namespace lake {
+namespace {
+constexpr int64_t kHostChunk = 1 << 20;
+
+size_t a256(size_t x) { return (x + 255) & ~(size_t)255; }
+
+struct SlotLayout {
+  size_t in, ids, dec, log, ws, total;
+};
+SlotLayout slot_layout(int64_t chunk, size_t in_b) {
+  SlotLayout L{};
+  size_t o = 0;
+  L.in = o; o += a256((size_t)chunk * in_b);
+  L.ids = o; o += a256((size_t)chunk * 4);
+  L.dec = o; o += a256((size_t)chunk);
+  L.log = o; o += a256((size_t)chunk * 8);
+  L.ws = o; o += a256(group_workspace_bytes(chunk));
+  L.total = o;
+  return L;
+}
+
+struct HostPipe {
+  bool init = false;
+  cudaStream_t h2d = nullptr, d2h = nullptr;
+  cudaEvent_t in_ready[2], comp_done[2], out_done[2];
+};
+std::mutex g_pipe_mu;
+HostPipe g_pipe[kMaxDevices];
+
+int pipe_for(int device, HostPipe **out) {
+  HostPipe &p = g_pipe[device];
+  if (!p.init) {
+    if (cudaStreamCreateWithFlags(&p.h2d, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaStreamCreateWithFlags(&p.d2h, cudaStreamNonBlocking) != cudaSuccess)
+      return LAKE_ERR_CUDA;
+    for (int i = 0; i < 2; ++i)
+      if (cudaEventCreateWithFlags(&p.in_ready[i], cudaEventDisableTiming) != cudaSuccess ||
+          cudaEventCreateWithFlags(&p.comp_done[i], cudaEventDisableTiming) != cudaSuccess ||
+          cudaEventCreateWithFlags(&p.out_done[i], cudaEventDisableTiming) != cudaSuccess)
+        return LAKE_ERR_CUDA;
+    p.init = true;
+  }
+  *out = &p;
+  return LAKE_OK;
+}
+}  // namespace
+}  // namespace lake
+
+extern "C" {
+
 size_t lake_linnos_host_staging_bytes(int64_t n, uint32_t flags) {
   if (n < 0) return 0;
   const size_t in_b = (flags & LAKE_IN_MASK) == LAKE_IN_RAW ? 36 : 32;
-  auto a = [](size_t x) { return (x + 255) & ~(size_t)255; };
-  return a((size_t)n * in_b) + a((size_t)n * 4) + a((size_t)n) + a((size_t)n * 8) +
-         a(group_workspace_bytes(n));
+  const int64_t chunk = n < kHostChunk ? (n > 0 ? n : 1) : kHostChunk;
+  return 2 * slot_layout(chunk, in_b).total;
 }
 
 int lake_linnos_infer_host(const void *h_in, uint32_t flags, int64_t n, int32_t model_id,
@@ -524,30 +578,72 @@ int lake_linnos_infer_host(const void *h_in, uint32_t flags, int64_t n, int32_t 
   if (n == 0) return LAKE_OK;
   if (!h_in || !h_decisions || !d_staging) return LAKE_ERR_INVAL;
   if (staging_bytes < lake_linnos_host_staging_bytes(n, flags)) return LAKE_ERR_NOMEM;
-  auto a = [](size_t x) { return (x + 255) & ~(size_t)255; };
-  const size_t in_b = in_kind == LAKE_IN_RAW ? 36 : 32;
-  uint8_t *p = static_cast<uint8_t *>(d_staging);
-  void *d_in = p; p += a((size_t)n * in_b);
-  int32_t *d_ids = reinterpret_cast<int32_t *>(p); p += a((size_t)n * 4);
-  uint8_t *d_dec = p; p += a((size_t)n);
-  float *d_log = reinterpret_cast<float *>(p); p += a((size_t)n * 8);
-  void *d_ws = p;
-  cudaStream_t s = static_cast<cudaStream_t>(stream);
-  cudaError_t e = cudaMemcpyAsync(d_in, h_in, (size_t)n * in_b, cudaMemcpyHostToDevice, s);
-  if (e != cudaSuccess) return cuda_status(e);
-  if (h_model_ids) {
-    e = cudaMemcpyAsync(d_ids, h_model_ids, (size_t)n * 4, cudaMemcpyHostToDevice, s);
-    if (e != cudaSuccess) return cuda_status(e);
-    rc = lake_linnos_infer_multi(d_in, flags, n, d_ids, d_dec, h_logits ? d_log : nullptr,
-                                 d_ws, a(group_workspace_bytes(n)), stream);
-  } else {
-    rc = lake_linnos_infer(d_in, flags, n, model_id, d_dec, h_logits ? d_log : nullptr, stream);
+  // AUTO decides on the whole batch, not per chunk
+  if ((flags & LAKE_PREC_MASK) == LAKE_PREC_AUTO)
+    flags = (flags & ~(uint32_t)LAKE_PREC_MASK) | (prec < 0 ? LAKE_PREC_FP32 : LAKE_PREC_F16);
+  int device;
+  if (cudaGetDevice(&device) != cudaSuccess) return LAKE_ERR_CUDA;
+  if (device < 0 || device >= kMaxDevices) return LAKE_ERR_INVAL;
+  if (!h_model_ids) {  // validate the single model once, before any copy
+    DevModel m;
+    rc = current_model(model_id, &device, &m, nullptr);
+    if (rc != LAKE_OK) return rc;
   }
+  std::lock_guard<std::mutex> lk(g_pipe_mu);
+  HostPipe *pp;
+  rc = pipe_for(device, &pp);
   if (rc != LAKE_OK) return rc;
-  e = cudaMemcpyAsync(h_decisions, d_dec, (size_t)n, cudaMemcpyDeviceToHost, s);
-  if (e == cudaSuccess && h_logits)
-    e = cudaMemcpyAsync(h_logits, d_log, (size_t)n * 8, cudaMemcpyDeviceToHost, s);
-  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  const size_t in_b = in_kind == LAKE_IN_RAW ? 36 : 32;
+  const int64_t chunk = n < kHostChunk ? n : kHostChunk;
+  const SlotLayout L = slot_layout(chunk, in_b);
+  const int64_t nchunks = (n + chunk - 1) / chunk;
+  uint8_t *base = static_cast<uint8_t *>(d_staging);
+  // the staging slots must not be overwritten while earlier work on `s` still uses them
+  cudaEvent_t start_ev;
+  if (cudaEventCreateWithFlags(&start_ev, cudaEventDisableTiming) != cudaSuccess)
+    return LAKE_ERR_CUDA;
+  cudaError_t e = cudaEventRecord(start_ev, s);
+  if (e == cudaSuccess) e = cudaStreamWaitEvent(pp->h2d, start_ev, 0);
+  for (int64_t c = 0; c < nchunks && e == cudaSuccess; ++c) {
+    const int slot = (int)(c & 1);
+    uint8_t *sb = base + slot * L.total;
+    const int64_t off = c * chunk;
+    const int64_t cn = (n - off) < chunk ? (n - off) : chunk;
+    if (c >= 2) e = cudaStreamWaitEvent(pp->h2d, pp->comp_done[slot], 0);  // input slot free
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(sb + L.in, static_cast<const uint8_t *>(h_in) + off * in_b, cn * in_b,
+                          cudaMemcpyHostToDevice, pp->h2d);
+    if (e == cudaSuccess && h_model_ids)
+      e = cudaMemcpyAsync(sb + L.ids, h_model_ids + off, cn * 4, cudaMemcpyHostToDevice, pp->h2d);
+    if (e == cudaSuccess) e = cudaEventRecord(pp->in_ready[slot], pp->h2d);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(s, pp->in_ready[slot], 0);
+    if (e == cudaSuccess && c >= 2) e = cudaStreamWaitEvent(s, pp->out_done[slot], 0);  // outputs read
+    if (e != cudaSuccess) break;
+    uint8_t *d_dec = sb + L.dec;
+    float *d_log = h_logits ? reinterpret_cast<float *>(sb + L.log) : nullptr;
+    if (h_model_ids)
+      rc = lake_linnos_infer_multi(sb + L.in, flags, cn, reinterpret_cast<int32_t *>(sb + L.ids),
+                                   d_dec, d_log, sb + L.ws, L.total - L.ws, stream);
+    else
+      rc = lake_linnos_infer(sb + L.in, flags, cn, model_id, d_dec, d_log, stream);
+    if (rc != LAKE_OK) break;
+    e = cudaEventRecord(pp->comp_done[slot], s);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(pp->d2h, pp->comp_done[slot], 0);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(h_decisions + off, d_dec, cn, cudaMemcpyDeviceToHost, pp->d2h);
+    if (e == cudaSuccess && h_logits)
+      e = cudaMemcpyAsync(h_logits + off * 2, d_log, cn * 8, cudaMemcpyDeviceToHost, pp->d2h);
+    if (e == cudaSuccess) e = cudaEventRecord(pp->out_done[slot], pp->d2h);
+  }
+  cudaError_t e2 = cudaStreamSynchronize(pp->h2d);
+  cudaError_t e3 = cudaStreamSynchronize(pp->d2h);
+  cudaError_t e4 = cudaStreamSynchronize(s);
+  cudaEventDestroy(start_ev);
+  if (rc != LAKE_OK) return rc;
+  if (e == cudaSuccess) e = e2;
+  if (e == cudaSuccess) e = e3;
+  if (e == cudaSuccess) e = e4;
   return cuda_status(e);
 }
 

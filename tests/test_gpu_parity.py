@@ -274,3 +274,37 @@ def test_c3_full_size_sampled(prec):
         met = tc_metrics(lg[smp], dec[smp], rlg, rdec)
         assert met["max_rel"] <= 2e-2 and met["max_disagree_margin"] < 5e-2, met
         assert met["agreement"] >= 0.999, met
+
+
+# ------------------------------------------------------------------------- host-buffer path
+def _host_call(raw, flags, model_id=-1, ids=None, logits=True):
+    import torch
+    n = raw.shape[0]
+    h_in = torch.from_numpy(np.ascontiguousarray(raw).view(np.int32)).pin_memory()
+    h_ids = torch.from_numpy(ids.astype(np.int32)).pin_memory() if ids is not None else None
+    h_dec = torch.full((n,), 7, dtype=torch.uint8).pin_memory()
+    h_lg = torch.full((n, 2), 1234.0, dtype=torch.float32).pin_memory() if logits else None
+    sb = lake.host_staging_bytes(n, flags)
+    stg = torch.empty(sb, dtype=torch.uint8, device="cuda:0")
+    lake.infer_host(h_in, flags, n, model_id, h_ids, h_dec, h_lg, stg, sb)
+    return (h_lg.numpy() if logits else None), h_dec.numpy()
+
+
+@pytest.mark.parametrize("prec", [lake.LAKE_PREC_F16, lake.LAKE_PREC_FP32])
+def test_infer_host_single_equals_device(prec):
+    raw = _trace(5000, seed=44)
+    lg, dec = _host_call(raw, lake.LAKE_IN_RAW | prec, model_id=12)
+    dlg, ddec = run_infer(12, raw, lake.LAKE_IN_RAW | prec)
+    assert np.array_equal(dec, ddec)
+    assert np.array_equal(lg.view(np.uint32), dlg.view(np.uint32))
+
+
+def test_infer_host_pipelined_multi_equals_device(many_models):
+    # > 2 chunks of 2^20 with a ragged tail: exercises the slot reuse of the pipeline
+    n = (1 << 21) + 54321
+    raw, mids = inputs.multi_device_trace(n, 6, seed_base=1900, rerate=3.0)
+    ids = np.array(list(many_models))[mids]
+    lg, dec = _host_call(raw, lake.LAKE_IN_RAW | lake.LAKE_PREC_F16, ids=ids)
+    dlg, ddec, _ = run_multi(raw, ids, lake.LAKE_IN_RAW | lake.LAKE_PREC_F16)
+    assert np.array_equal(dec, ddec)
+    assert np.array_equal(lg.view(np.uint32), dlg.view(np.uint32))
