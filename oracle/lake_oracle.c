@@ -113,11 +113,11 @@ int oracle_mlp(int n_layers, const int *widths, const float *blob, const float *
         if (widths[l] > maxw) maxw = widths[l];
     }
 #ifdef _OPENMP
-    if (nthreads > 0) omp_set_num_threads(nthreads);
+    const int nt = nthreads > 0 ? nthreads : omp_get_num_procs();  /* no global OpenMP state */
 #else
     (void)nthreads;
 #endif
-#pragma omp parallel for schedule(static)
+#pragma omp parallel for schedule(static) num_threads(nt)
     for (int64_t i = 0; i < n; ++i) {
         float bufa[maxw], bufb[maxw];            /* C99 VLAs: per-I/O activations */
         float *h = bufa, *hn = bufb;
@@ -186,7 +186,7 @@ int oracle_infer_digits(int arch, const float *blob, const uint8_t *digits31, in
 int oracle_max_threads(void)
 {
 #ifdef _OPENMP
-    return omp_get_max_threads();
+    return omp_get_num_procs();
 #else
     return 1;
 #endif

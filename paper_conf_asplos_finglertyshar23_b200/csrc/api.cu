@@ -535,7 +535,7 @@ SlotLayout slot_layout(int64_t chunk, size_t in_b) {
 struct HostPipe {
   bool init = false;
   cudaStream_t h2d = nullptr, d2h = nullptr;
-  cudaEvent_t in_ready[2], comp_done[2], out_done[2];
+  cudaEvent_t start, in_ready[2], comp_done[2], out_done[2];
 };
 std::mutex g_pipe_mu;
 HostPipe g_pipe[kMaxDevices];
@@ -545,6 +545,8 @@ int pipe_for(int device, HostPipe **out) {
   if (!p.init) {
     if (cudaStreamCreateWithFlags(&p.h2d, cudaStreamNonBlocking) != cudaSuccess ||
         cudaStreamCreateWithFlags(&p.d2h, cudaStreamNonBlocking) != cudaSuccess)
+      return LAKE_ERR_CUDA;
+    if (cudaEventCreateWithFlags(&p.start, cudaEventDisableTiming) != cudaSuccess)
       return LAKE_ERR_CUDA;
     for (int i = 0; i < 2; ++i)
       if (cudaEventCreateWithFlags(&p.in_ready[i], cudaEventDisableTiming) != cudaSuccess ||
@@ -600,11 +602,8 @@ int lake_linnos_infer_host(const void *h_in, uint32_t flags, int64_t n, int32_t 
   const int64_t nchunks = (n + chunk - 1) / chunk;
   uint8_t *base = static_cast<uint8_t *>(d_staging);
   // the staging slots must not be overwritten while earlier work on `s` still uses them
-  cudaEvent_t start_ev;
-  if (cudaEventCreateWithFlags(&start_ev, cudaEventDisableTiming) != cudaSuccess)
-    return LAKE_ERR_CUDA;
-  cudaError_t e = cudaEventRecord(start_ev, s);
-  if (e == cudaSuccess) e = cudaStreamWaitEvent(pp->h2d, start_ev, 0);
+  cudaError_t e = cudaEventRecord(pp->start, s);
+  if (e == cudaSuccess) e = cudaStreamWaitEvent(pp->h2d, pp->start, 0);
   for (int64_t c = 0; c < nchunks && e == cudaSuccess; ++c) {
     const int slot = (int)(c & 1);
     uint8_t *sb = base + slot * L.total;
@@ -639,7 +638,6 @@ int lake_linnos_infer_host(const void *h_in, uint32_t flags, int64_t n, int32_t 
   cudaError_t e2 = cudaStreamSynchronize(pp->h2d);
   cudaError_t e3 = cudaStreamSynchronize(pp->d2h);
   cudaError_t e4 = cudaStreamSynchronize(s);
-  cudaEventDestroy(start_ev);
   if (rc != LAKE_OK) return rc;
   if (e == cudaSuccess) e = e2;
   if (e == cudaSuccess) e = e3;

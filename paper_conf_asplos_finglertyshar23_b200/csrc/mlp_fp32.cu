@@ -6,8 +6,10 @@
 // Network: "two layers with 256 and 2 neurons" (+1 / +2 hidden layers), §7.1
 // P:1168-1177. Batch scoring (score_features, Table 1).
 //
-// Mapping: a CTA (256 threads) owns a 64-I/O tile. Hidden layers are register-tiled GEMMs:
-// thread (tr = warp, tc = lane) owns 8 rows {tr*4+i, 32+tr*4+i} x 8 columns {tc + 32*jj}.
+// Mapping: a CTA (256 threads) owns an M-I/O tile (M = 64, or 16 for small single-model
+// batches, where latency rather than throughput matters). Hidden layers are register-tiled
+// GEMMs: thread (tr = warp, tc = lane) owns RM = M/8 rows {h*M/2 + tr*RM/2 + i} x 8 columns
+// {tc + 32*jj}.
 // Each accumulator is summed over k strictly in order (that is what a K-loop GEMM does),
 // so the tiling changes nothing numerically. Activations live transposed in SMEM
 // (act[k][row], row stride 68 floats: broadcast A reads, conflict-free epilogue stores);
@@ -22,16 +24,24 @@
 namespace lake {
 namespace {
 
-constexpr int M = kF32TileM;
-constexpr int S = kF32ActStride;
 constexpr int KC = kF32KChunk;
 
+template <int RM>
+struct F32Cfg {
+  static constexpr int M = 8 * RM;                       // rows per tile
+  static constexpr int HR = RM / 2;                      // rows per thread per half-tile
+  // activation row stride: float4-aligned with a 4-float pad for RM = 8 (conflict-free
+  // float4 epilogue stores), odd for RM = 2 (conflict-free scalar stores)
+  static constexpr int S = RM == 8 ? kF32ActStride : M + 1;
+};
+
+template <int RM>
 struct F32Smem {
-  float act[2][kHidden][S];     // transposed activations, ping-pong
-  float w[2][KC][kHidden];      // W^T chunk staging (permuted columns)
+  float act[2][kHidden][F32Cfg<RM>::S];  // transposed activations, ping-pong
+  float w[2][KC][kHidden];               // W^T chunk staging (permuted columns)
   float wout[2][kHidden];
   float bout[4];
-  int32_t rows[M];              // I/O index per tile row, -1 = padding
+  int32_t rows[F32Cfg<RM>::M];           // I/O index per tile row, -1 = padding
 };
 
 __device__ __forceinline__ void stage_chunk(float (*dst)[kHidden], const float *src, int rows) {
@@ -44,13 +54,14 @@ __device__ __forceinline__ void stage_chunk(float (*dst)[kHidden], const float *
   __pipeline_commit();
 }
 
-template <int IN_KIND>
+template <int IN_KIND, int RM>
 __global__ void __launch_bounds__(kF32Threads, 1)
 mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
                 uint8_t *__restrict__ decisions,
                 float *__restrict__ logits) {
+  constexpr int M = F32Cfg<RM>::M, S = F32Cfg<RM>::S, HR = F32Cfg<RM>::HR;
   extern __shared__ __align__(16) uint8_t smem_raw[];
-  F32Smem &sm = *reinterpret_cast<F32Smem *>(smem_raw);
+  F32Smem<RM> &sm = *reinterpret_cast<F32Smem<RM> *>(smem_raw);
   const int tid = threadIdx.x;
   const int tr = tid >> 5;   // warp: row group
   const int tc = tid & 31;   // lane: column group
@@ -110,9 +121,9 @@ mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched t
       const float *wt = mp->wt[l];
       const float (*ain)[S] = sm.act[l & 1];
       float (*aout)[S] = sm.act[(l + 1) & 1];
-      float acc[8][8];
+      float acc[RM][8];
 #pragma unroll
-      for (int i = 0; i < 8; ++i)
+      for (int i = 0; i < RM; ++i)
 #pragma unroll
         for (int j = 0; j < 8; ++j) acc[i][j] = 0.0f;
       const int nch = Kst / KC;
@@ -130,14 +141,24 @@ mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched t
 #pragma unroll 4
         for (int kk = 0; kk < kmax; ++kk) {
           const int k = c * KC + kk;
-          const float4 a0 = *reinterpret_cast<const float4 *>(&ain[k][tr * 4]);
-          const float4 a1 = *reinterpret_cast<const float4 *>(&ain[k][32 + tr * 4]);
+          float av[RM];
+          if constexpr (HR == 4) {
+            const float4 a0 = *reinterpret_cast<const float4 *>(&ain[k][tr * 4]);
+            const float4 a1 = *reinterpret_cast<const float4 *>(&ain[k][M / 2 + tr * 4]);
+            av[0] = a0.x; av[1] = a0.y; av[2] = a0.z; av[3] = a0.w;
+            av[4] = a1.x; av[5] = a1.y; av[6] = a1.z; av[7] = a1.w;
+          } else {
+#pragma unroll
+            for (int i = 0; i < HR; ++i) {
+              av[i] = ain[k][tr * HR + i];
+              av[HR + i] = ain[k][M / 2 + tr * HR + i];
+            }
+          }
           const float4 b0 = *reinterpret_cast<const float4 *>(&wc[kk][tc * 4]);
           const float4 b1 = *reinterpret_cast<const float4 *>(&wc[kk][128 + tc * 4]);
-          const float av[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
           const float bv[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
 #pragma unroll
-          for (int i = 0; i < 8; ++i)
+          for (int i = 0; i < RM; ++i)
 #pragma unroll
             for (int j = 0; j < 8; ++j) acc[i][j] = __fmaf_rn(av[i], bv[j], acc[i][j]);
         }
@@ -149,14 +170,23 @@ mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched t
       for (int jj = 0; jj < 8; ++jj) {
         const int j = tc + 32 * jj;
         const float bj = __ldg(bias + j);
-        float h[8];
+        float h[RM];
 #pragma unroll
-        for (int i = 0; i < 8; ++i) {
+        for (int i = 0; i < RM; ++i) {
           const float z = __fadd_rn(acc[i][jj], bj);
           h[i] = (z > 0.0f) ? z : 0.0f;
         }
-        *reinterpret_cast<float4 *>(&aout[j][tr * 4]) = make_float4(h[0], h[1], h[2], h[3]);
-        *reinterpret_cast<float4 *>(&aout[j][32 + tr * 4]) = make_float4(h[4], h[5], h[6], h[7]);
+        if constexpr (HR == 4) {
+          *reinterpret_cast<float4 *>(&aout[j][tr * 4]) = make_float4(h[0], h[1], h[2], h[3]);
+          *reinterpret_cast<float4 *>(&aout[j][M / 2 + tr * 4]) =
+              make_float4(h[4], h[5], h[6], h[7]);
+        } else {
+#pragma unroll
+          for (int i = 0; i < HR; ++i) {
+            aout[j][tr * HR + i] = h[i];
+            aout[j][M / 2 + tr * HR + i] = h[HR + i];
+          }
+        }
       }
       __syncthreads();
     }
@@ -178,31 +208,49 @@ mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched t
   }
 }
 
+template <int IN_KIND, int RM>
+cudaError_t launch_rm(const void *in, const TileSched &ts, uint8_t *decisions, float *logits,
+                      cudaStream_t s, int64_t grid) {
+  const size_t smem = sizeof(F32Smem<RM>);
+  static bool attr_set[64] = {};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (!attr_set[dev & 63]) {
+    cudaError_t e = cudaFuncSetAttribute(mlp_fp32_kernel<IN_KIND, RM>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    attr_set[dev & 63] = true;
+  }
+  mlp_fp32_kernel<IN_KIND, RM><<<(unsigned)grid, kF32Threads, smem, s>>>(in, ts, decisions,
+                                                                       logits);
+  return cudaGetLastError();
+}
+
 }  // namespace
 
-cudaError_t launch_mlp_fp32(const void *in, int in_kind, const TileSched &ts,
+cudaError_t launch_mlp_fp32(const void *in, int in_kind, const TileSched &ts_in,
                             uint8_t *decisions, float *logits, cudaStream_t s, int device) {
-  int sms = 148;
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
-  const size_t smem = sizeof(F32Smem);
+  static int sms_cache[64] = {};
+  int sms = sms_cache[device & 63];
+  if (!sms) {
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+    sms_cache[device & 63] = sms;
+  }
+  TileSched ts = ts_in;
+  // small single-model batches: 16-row tiles (4x less work per tile on the critical path)
+  const bool small = ts.tile_model == nullptr && ts.n <= (int64_t)16 * sms;
+  if (small) ts.n_tiles = (ts.n + 15) / 16;
   const int64_t grid = ts.n_tiles < sms ? ts.n_tiles : sms;
   if (grid <= 0) return cudaSuccess;
   cudaError_t e;
-  if (in_kind == LAKE_IN_RAW) {
-    e = cudaFuncSetAttribute(mlp_fp32_kernel<LAKE_IN_RAW>,
-                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    mlp_fp32_kernel<LAKE_IN_RAW><<<(unsigned)grid, kF32Threads, smem, s>>>(in, ts, decisions,
-                                                                            logits);
-  } else {
-    e = cudaFuncSetAttribute(mlp_fp32_kernel<LAKE_IN_DIGITS>,
-                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    mlp_fp32_kernel<LAKE_IN_DIGITS><<<(unsigned)grid, kF32Threads, smem, s>>>(
-        in, ts, decisions, logits);
-  }
+  if (in_kind == LAKE_IN_RAW)
+    e = small ? launch_rm<LAKE_IN_RAW, 2>(in, ts, decisions, logits, s, grid)
+              : launch_rm<LAKE_IN_RAW, 8>(in, ts, decisions, logits, s, grid);
+  else
+    e = small ? launch_rm<LAKE_IN_DIGITS, 2>(in, ts, decisions, logits, s, grid)
+              : launch_rm<LAKE_IN_DIGITS, 8>(in, ts, decisions, logits, s, grid);
   count_launch();
-  return cudaGetLastError();
+  return e;
 }
 
 }  // namespace lake

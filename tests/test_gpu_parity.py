@@ -18,7 +18,7 @@ from paper_conf_asplos_finglertyshar23_b200 import inputs, lake
 pytestmark = pytest.mark.gpu
 
 ARCHS = [0, 1, 2]
-RAGGED = [1, 63, 64, 65, 255, 257, 1000, 4096 + 17]
+RAGGED = [1, 15, 17, 63, 64, 65, 255, 257, 1000, 2368, 2369, 4096 + 17]  # FP32: 16-row tiles up to 16*148
 
 
 @pytest.fixture(scope="module", autouse=True)
