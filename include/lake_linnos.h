@@ -178,7 +178,10 @@ int lake_linnos_multi_status(const void *workspace, size_t ws_bytes, int64_t *n_
  * h_logits != NULL) on a second internal stream, so chunk i+1's upload and chunk i-1's
  * download overlap chunk i's kernels. Synchronous: returns when every output is on the host.
  * d_staging: device buffer of at least lake_linnos_host_staging_bytes(n, flags) bytes (two
- * chunk slots). LAKE_PREC_AUTO is resolved once for the whole batch. */
+ * chunk slots). LAKE_PREC_AUTO is resolved once for the whole batch. Batches of at most
+ * 2^14 I/Os whose host buffers are all pinned and mapped (cudaHostAlloc / cudaHostRegister
+ * under UVA) skip the copies: the kernel reads and writes host memory directly (zero-copy),
+ * which is what bounds small-batch latency (Fig. 8's batch sizes). */
 size_t lake_linnos_host_staging_bytes(int64_t n, uint32_t flags);
 int lake_linnos_infer_host(const void *h_in, uint32_t flags, int64_t n, int32_t model_id,
                            const int32_t *h_model_ids, uint8_t *h_decisions, float *h_logits,

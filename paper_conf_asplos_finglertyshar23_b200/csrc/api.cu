@@ -514,6 +514,18 @@ int lake_linnos_multi_status(const void *workspace, size_t ws_bytes, int64_t *n_
 namespace lake {
 namespace {
 constexpr int64_t kHostChunk = 1 << 20;
+constexpr int64_t kZeroCopyMax = 1 << 14;
+
+// Device-accessible alias of a pinned, mapped host pointer (UVA), or nullptr.
+void *mapped(const void *h) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, h) != cudaSuccess) {
+    cudaGetLastError();  // pageable memory on older drivers reports an error: clear it
+    return nullptr;
+  }
+  if (a.type != cudaMemoryTypeHost || a.devicePointer == nullptr) return nullptr;
+  return a.devicePointer;
+}
 
 size_t a256(size_t x) { return (x + 255) & ~(size_t)255; }
 
@@ -591,16 +603,55 @@ int lake_linnos_infer_host(const void *h_in, uint32_t flags, int64_t n, int32_t 
     rc = current_model(model_id, &device, &m, nullptr);
     if (rc != LAKE_OK) return rc;
   }
-  std::lock_guard<std::mutex> lk(g_pipe_mu);
-  HostPipe *pp;
-  rc = pipe_for(device, &pp);
-  if (rc != LAKE_OK) return rc;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   const size_t in_b = in_kind == LAKE_IN_RAW ? 36 : 32;
   const int64_t chunk = n < kHostChunk ? n : kHostChunk;
   const SlotLayout L = slot_layout(chunk, in_b);
   const int64_t nchunks = (n + chunk - 1) / chunk;
   uint8_t *base = static_cast<uint8_t *>(d_staging);
+  if (n <= kZeroCopyMax) {
+    // small batch: if every host buffer is pinned and mapped (UVA), the fused kernel reads
+    // the records from and writes the decisions to host memory directly - no copy-engine
+    // round trips (they, not the kernel, dominate the latency of a small batch)
+    void *d_in = mapped(h_in), *d_dec = mapped(h_decisions);
+    void *d_ids = h_model_ids ? mapped(h_model_ids) : nullptr;
+    void *d_log = h_logits ? mapped(h_logits) : nullptr;
+    if (d_in && d_dec && (!h_model_ids || d_ids) && (!h_logits || d_log)) {
+      if (h_model_ids)
+        rc = lake_linnos_infer_multi(d_in, flags, n, static_cast<int32_t *>(d_ids),
+                                     static_cast<uint8_t *>(d_dec), static_cast<float *>(d_log),
+                                     base + L.ws, L.total - L.ws, stream);
+      else
+        rc = lake_linnos_infer(d_in, flags, n, model_id, static_cast<uint8_t *>(d_dec),
+                               static_cast<float *>(d_log), stream);
+      if (rc != LAKE_OK) return rc;
+      return cuda_status(cudaStreamSynchronize(s));
+    }
+  }
+  if (nchunks == 1) {
+    // one chunk: nothing to overlap, so stay on the caller's stream (no cross-stream hops)
+    cudaError_t e = cudaMemcpyAsync(base + L.in, h_in, n * in_b, cudaMemcpyHostToDevice, s);
+    if (e == cudaSuccess && h_model_ids)
+      e = cudaMemcpyAsync(base + L.ids, h_model_ids, n * 4, cudaMemcpyHostToDevice, s);
+    if (e != cudaSuccess) return cuda_status(e);
+    uint8_t *d_dec = base + L.dec;
+    float *d_log = h_logits ? reinterpret_cast<float *>(base + L.log) : nullptr;
+    if (h_model_ids)
+      rc = lake_linnos_infer_multi(base + L.in, flags, n, reinterpret_cast<int32_t *>(base + L.ids),
+                                   d_dec, d_log, base + L.ws, L.total - L.ws, stream);
+    else
+      rc = lake_linnos_infer(base + L.in, flags, n, model_id, d_dec, d_log, stream);
+    if (rc != LAKE_OK) return rc;
+    e = cudaMemcpyAsync(h_decisions, d_dec, n, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess && h_logits)
+      e = cudaMemcpyAsync(h_logits, d_log, n * 8, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    return cuda_status(e);
+  }
+  std::lock_guard<std::mutex> lk(g_pipe_mu);
+  HostPipe *pp;
+  rc = pipe_for(device, &pp);
+  if (rc != LAKE_OK) return rc;
   // the staging slots must not be overwritten while earlier work on `s` still uses them
   cudaError_t e = cudaEventRecord(pp->start, s);
   if (e == cudaSuccess) e = cudaStreamWaitEvent(pp->h2d, pp->start, 0);
