@@ -76,7 +76,20 @@ constexpr uint32_t kEpiWarps = 4 * kEpiPerQ;       // 16
 #endif
 constexpr uint32_t kChunks = LAKE_CHUNKS;          // H column chunks per layer (MMA K-chunks)
 constexpr uint32_t kChunkCols = kHidden / kChunks;
-constexpr uint32_t kEpiCols = kChunkCols / kEpiPerQ;  // columns per warp per chunk
+#ifdef LAKE_EPI_INTERLEAVE
+// warp hh of a quadrant converts chunks hh, hh+kEpiPerQ, ... (all columns of each), so
+// consecutive chunks are produced concurrently by different warps
+constexpr bool kInterleave = true;
+constexpr uint32_t kEpiCols = kChunkCols;              // columns per warp per chunk
+constexpr uint32_t kWarpChunks = kChunks / kEpiPerQ;   // chunks per warp per layer
+constexpr uint32_t kHreadyCount = 2 * 4;               // one warp per quadrant, both CTAs
+#else
+// the kEpiPerQ warps of a quadrant split every chunk's columns between them
+constexpr bool kInterleave = false;
+constexpr uint32_t kEpiCols = kChunkCols / kEpiPerQ;
+constexpr uint32_t kWarpChunks = kChunks;
+constexpr uint32_t kHreadyCount = 2 * kEpiWarps;
+#endif
 constexpr uint32_t kKStepsPerChunk = kChunkCols / 16;
 constexpr int kThreads = 32 * (3 + kEpiWarps + 1);  // digitisers(2) + loader + epi + MMA
 constexpr uint32_t kHBytes = 128 * kHidden * 2;   // 64 KB
@@ -234,7 +247,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       ptx::mbar_init(bar(B_DFULL + i), 1);       // tcgen05.commit (multicast)
       ptx::mbar_init(bar(B_TEMPTY + i), 2 * kEpiWarps);  // every epilogue warp, both CTAs
     }
-    for (uint32_t i = 0; i < kChunks; ++i) ptx::mbar_init(bar(B_HREADY + i), 2 * kEpiWarps);
+    for (uint32_t i = 0; i < kChunks; ++i) ptx::mbar_init(bar(B_HREADY + i), kHreadyCount);
     ptx::mbar_init(bar(B_WFREE), 1);             // tcgen05.commit (multicast)
     ptx::fence_mbar_init();
   }
@@ -477,29 +490,37 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         d_phase ^= (1u << b);
         LAKE_TEV(T_DFULL, it, l, warp);
         ptx::tc_fence_after();
-        const uint32_t tbase = tmem + ((q * 32) << 16) + b * 256 + hh * W;
+        const uint32_t tbase = tmem + ((q * 32) << 16) + b * 256;
+        // j-th (chunk, first column) handled by this warp
+        auto chunk_of = [&](uint32_t j) { return kInterleave ? j * kEpiPerQ + hh : j; };
+        auto col_of = [&](uint32_t j) {
+          return kInterleave ? chunk_of(j) * kChunkCols : j * kChunkCols + hh * W;
+        };
         const float *bl = prm + l * kHidden;
+#ifdef LAKE_NO_EPI_PREFETCH
+        constexpr bool kPrefetch = false;
+#else
         constexpr bool kPrefetch = W <= 32;  // two W-register buffers
+#endif
         uint32_t ra[W], rb[W];  // rb unused (eliminated) without prefetch
-        (void)rb;
-        ptx::tmem_ld_cols<W>(tbase, ra);
+        ptx::tmem_ld_cols<W>(tbase + col_of(0), ra);
         ptx::tmem_ld_wait();
         if (l + 1 < nh) {
-          // hidden layer feeding another MMA: kChunks chunks; with two register buffers the
-          // TMEM load of chunk kc+1 is in flight while chunk kc is converted and stored
+          // hidden layer feeding another MMA; with two register buffers the TMEM load of the
+          // warp's next chunk is in flight while the current one is converted and stored
 #pragma unroll
-          for (uint32_t kc = 0; kc < kChunks; ++kc) {
-            const uint32_t col0 = kc * kChunkCols + hh * W;
+          for (uint32_t j = 0; j < kWarpChunks; ++j) {
+            const uint32_t kc = chunk_of(j), col0 = col_of(j);
             if constexpr (kPrefetch) {
-              if (kc + 1 < kChunks) {
-                if (kc & 1) ptx::tmem_ld_cols<W>(tbase + (kc + 1) * kChunkCols, ra);
-                else ptx::tmem_ld_cols<W>(tbase + (kc + 1) * kChunkCols, rb);
+              if (j + 1 < kWarpChunks) {
+                if (j & 1) ptx::tmem_ld_cols<W>(tbase + col_of(j + 1), ra);
+                else ptx::tmem_ld_cols<W>(tbase + col_of(j + 1), rb);
               }
-              if (kc & 1) epi_to_h<PREC, W>(rb, prm2 + l * kHidden / 2, col0, hrow);
+              if (j & 1) epi_to_h<PREC, W>(rb, prm2 + l * kHidden / 2, col0, hrow);
               else epi_to_h<PREC, W>(ra, prm2 + l * kHidden / 2, col0, hrow);
             } else {
-              if (kc > 0) {
-                ptx::tmem_ld_cols<W>(tbase + kc * kChunkCols, ra);
+              if (j > 0) {
+                ptx::tmem_ld_cols<W>(tbase + col0, ra);
                 ptx::tmem_ld_wait();
               }
               epi_to_h<PREC, W>(ra, prm2 + l * kHidden / 2, col0, hrow);
@@ -510,26 +531,26 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
             __syncwarp();
             if (lane == 0) ptx::mbar_arrive_cluster(hready_leader0 + kc * 8);
             LAKE_TEV(T_CHUNK, it, l, kc);
-            if (kPrefetch && kc + 1 < kChunks) ptx::tmem_ld_wait();
+            if (kPrefetch && j + 1 < kWarpChunks) ptx::tmem_ld_wait();
             LAKE_TEV(T_LDWAIT, it, l, kc);
           }
         } else {
           // last hidden layer: fold the 2-neuron output layer (fp32, CUDA cores)
           float p[4] = {0.0f, 0.0f, 0.0f, 0.0f};
 #pragma unroll
-          for (uint32_t kc = 0; kc < kChunks; ++kc) {
-            const uint32_t col0 = kc * kChunkCols + hh * W;
+          for (uint32_t j = 0; j < kWarpChunks; ++j) {
+            const uint32_t col0 = col_of(j);
             if constexpr (kPrefetch) {
-              if (kc + 1 < kChunks) {
-                if (kc & 1) ptx::tmem_ld_cols<W>(tbase + (kc + 1) * kChunkCols, ra);
-                else ptx::tmem_ld_cols<W>(tbase + (kc + 1) * kChunkCols, rb);
+              if (j + 1 < kWarpChunks) {
+                if (j & 1) ptx::tmem_ld_cols<W>(tbase + col_of(j + 1), ra);
+                else ptx::tmem_ld_cols<W>(tbase + col_of(j + 1), rb);
               }
-              if (kc & 1) epi_to_logits<W>(rb, bl, wo, col0, p);
+              if (j & 1) epi_to_logits<W>(rb, bl, wo, col0, p);
               else epi_to_logits<W>(ra, bl, wo, col0, p);
-              if (kc + 1 < kChunks) ptx::tmem_ld_wait();
+              if (j + 1 < kWarpChunks) ptx::tmem_ld_wait();
             } else {
-              if (kc > 0) {
-                ptx::tmem_ld_cols<W>(tbase + kc * kChunkCols, ra);
+              if (j > 0) {
+                ptx::tmem_ld_cols<W>(tbase + col0, ra);
                 ptx::tmem_ld_wait();
               }
               epi_to_logits<W>(ra, bl, wo, col0, p);
