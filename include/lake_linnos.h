@@ -187,6 +187,24 @@ int lake_linnos_infer_host(const void *h_in, uint32_t flags, int64_t n, int32_t 
                            const int32_t *h_model_ids, uint8_t *h_decisions, float *h_logits,
                            void *d_staging, size_t staging_bytes, void *stream);
 
+/* GPU feature capture: the raw records the feature registry would
+ * capture on issue and completion (Fig. 4 / Fig. 5), computed for a whole trace.
+ * Inputs (device pointers, n entries, any order): arrival_ns[i], complete_ns[i] (int64, ns,
+ * 0 <= arrival < complete < 2^47) and device[i] (int32 in [0, 65535]; NULL = one device).
+ * Output raw_out[i] (lake_io_raw_t, device memory), with DESIGN.md readings R7-R10:
+ *   q_now     = I/Os of the same device issued at or before i (ties in arrival by index,
+ *               i included) that complete after a_i; an I/O completing exactly at a_i counts
+ *               as completed;
+ *   history k = the k-th newest completed I/O of the device by (complete_ns, index):
+ *               lat_us = floor((complete - arrival) / 1000) (clamped to uint32), q_hist =
+ *               its own q_now; zeros when fewer than k+1 have completed.
+ * workspace: device buffer of lake_linnos_capture_workspace_bytes(n) bytes (else
+ * LAKE_ERR_NOMEM). Asynchronous on `stream`; n <= INT32_MAX. Bit-exact (integer). */
+size_t lake_linnos_capture_workspace_bytes(int64_t n);
+int lake_linnos_capture(const int64_t *arrival_ns, const int64_t *complete_ns,
+                        const int32_t *device, int64_t n, lake_io_raw_t *raw_out,
+                        void *workspace, size_t ws_bytes, void *stream);
+
 /* Number of kernels this library launched on the current device since the last reset
  * (host-side counter; used by the bench to report gpu_launches). */
 uint64_t lake_linnos_launch_count(void);

@@ -11,6 +11,8 @@ citations and readings). Parity status per function:
 * ``digitize``              pinned (hand-worked golden examples, brute-force round trip)
 * ``mlp`` / ``infer_raw``   pinned (tiny integer MLPs vs int64, IEEE order examples,
                              invariants, numpy float64 GEMM chain)
+* ``capture``               pinned (hand-worked trace, heap-based event simulation of the
+                             generator, invariants)
 * parity against the paper's trained model: unpinned (no weights/traces published).
 """
 from __future__ import annotations
@@ -56,6 +58,10 @@ def _load():
         lib.oracle_infer_digits.argtypes = [ctypes.c_int, P, P, ctypes.c_int64, P, P,
                                             ctypes.c_int]
         lib.oracle_infer_digits.restype = ctypes.c_int
+        lib.oracle_capture.argtypes = [P, P, P, ctypes.c_int64, P]
+        lib.oracle_capture.restype = None
+        lib.oracle_capture_rows.argtypes = [P, P, P, ctypes.c_int64, P, ctypes.c_int64, P]
+        lib.oracle_capture_rows.restype = None
         lib.oracle_max_threads.argtypes = []
         lib.oracle_max_threads.restype = ctypes.c_int
         _lib = lib
@@ -140,3 +146,26 @@ def infer_multi_raw(models: dict, raw: np.ndarray, model_ids: np.ndarray, nthrea
         logits[idx] = lg
         dec[idx] = d
     return logits, dec
+
+
+def capture(arrival_ns: np.ndarray, complete_ns: np.ndarray, device=None) -> np.ndarray:
+    """Feature capture (NEXT-1): per-I/O raw records uint32[n, 9] from a trace."""
+    a = np.ascontiguousarray(arrival_ns, dtype=np.int64)
+    c = np.ascontiguousarray(complete_ns, dtype=np.int64)
+    n = a.shape[0]
+    out = np.zeros((n, 9), dtype=np.uint32)
+    d = None if device is None else np.ascontiguousarray(device, dtype=np.int32)
+    _load().oracle_capture(_ptr(a), _ptr(c), None if d is None else _ptr(d), n, _ptr(out))
+    return out
+
+
+def capture_rows(arrival_ns, complete_ns, device, rows) -> np.ndarray:
+    """capture() for selected rows only (O(n) per row): uint32[len(rows), 9]."""
+    a = np.ascontiguousarray(arrival_ns, dtype=np.int64)
+    c = np.ascontiguousarray(complete_ns, dtype=np.int64)
+    r = np.ascontiguousarray(rows, dtype=np.int64)
+    out = np.zeros((r.shape[0], 9), dtype=np.uint32)
+    d = None if device is None else np.ascontiguousarray(device, dtype=np.int32)
+    _load().oracle_capture_rows(_ptr(a), _ptr(c), None if d is None else _ptr(d), a.shape[0],
+                                _ptr(r), r.shape[0], _ptr(out))
+    return out

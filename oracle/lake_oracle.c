@@ -183,6 +183,103 @@ int oracle_infer_digits(int arch, const float *blob, const uint8_t *digits31, in
     return rc;
 }
 
+/*
+ * Feature capture (NEXT-1; Fig. 4/5 P:861-932; readings R7-R10), the plain definition.
+ * I/O i of device d (arrival a_i, completion c_i, both ns):
+ *   q_now_i   = #{ j of d : (a_j, j) <= (a_i, i) and c_j > a_i }        (pending incl. self)
+ *   C_i       = { j of d : c_j <= a_i }                                   (completed at issue)
+ *   history   = the 4 largest members of C_i by (c_j, j); [0] = most recent
+ *   lat_us[k] = floor((c_j - a_j) / 1000) (clamped to uint32), q_hist[k] = q_now_j; else 0.
+ * dev may be NULL (one device). O(n^2): test sizes only. raw_out: uint32[n][9].
+ */
+void oracle_capture(const int64_t *a, const int64_t *c, const int32_t *dev, int64_t n,
+                    uint32_t *raw_out)
+{
+    uint32_t *q = (uint32_t *)malloc(sizeof(uint32_t) * (size_t)(n > 0 ? n : 1));
+    if (!q) return;
+    for (int64_t i = 0; i < n; ++i) {
+        uint32_t cnt = 0;
+        for (int64_t j = 0; j < n; ++j) {
+            if (dev && dev[j] != dev[i]) continue;
+            int issued_before = (a[j] < a[i]) || (a[j] == a[i] && j <= i);
+            if (issued_before && c[j] > a[i]) ++cnt;
+        }
+        q[i] = cnt;
+    }
+    for (int64_t i = 0; i < n; ++i) {
+        int64_t top[4] = {-1, -1, -1, -1};   /* top[0] = largest (c_j, j) */
+        for (int64_t j = 0; j < n; ++j) {
+            if (dev && dev[j] != dev[i]) continue;
+            if (c[j] > a[i]) continue;
+            for (int k = 0; k < 4; ++k) {
+                int64_t t = top[k];
+                if (t < 0 || c[j] > c[t] || (c[j] == c[t] && j > t)) {
+                    for (int m = 3; m > k; --m) top[m] = top[m - 1];
+                    top[k] = j;
+                    break;
+                }
+            }
+        }
+        uint32_t *r = raw_out + 9 * i;
+        r[0] = q[i];
+        for (int k = 0; k < 4; ++k) {
+            if (top[k] >= 0) {
+                int64_t us = (c[top[k]] - a[top[k]]) / 1000;
+                r[1 + k] = us > 0xFFFFFFFFLL ? 0xFFFFFFFFu : (uint32_t)us;
+                r[5 + k] = q[top[k]];
+            } else {
+                r[1 + k] = 0;
+                r[5 + k] = 0;
+            }
+        }
+    }
+    free(q);
+}
+
+/* Same definition for selected rows only (O(n) per row): raw_out uint32[m][9] for rows[]. */
+void oracle_capture_rows(const int64_t *a, const int64_t *c, const int32_t *dev, int64_t n,
+                         const int64_t *rows, int64_t m, uint32_t *raw_out)
+{
+    for (int64_t r = 0; r < m; ++r) {
+        const int64_t i = rows[r];
+        uint32_t q = 0;
+        int64_t top[4] = {-1, -1, -1, -1};
+        for (int64_t j = 0; j < n; ++j) {
+            if (dev && dev[j] != dev[i]) continue;
+            int issued_before = (a[j] < a[i]) || (a[j] == a[i] && j <= i);
+            if (issued_before && c[j] > a[i]) ++q;
+            if (c[j] > a[i]) continue;
+            for (int k = 0; k < 4; ++k) {
+                int64_t t = top[k];
+                if (t < 0 || c[j] > c[t] || (c[j] == c[t] && j > t)) {
+                    for (int mm = 3; mm > k; --mm) top[mm] = top[mm - 1];
+                    top[k] = j;
+                    break;
+                }
+            }
+        }
+        uint32_t *o = raw_out + 9 * r;
+        o[0] = q;
+        for (int k = 0; k < 4; ++k) {
+            if (top[k] >= 0) {
+                const int64_t j = top[k];
+                int64_t us = (c[j] - a[j]) / 1000;
+                o[1 + k] = us > 0xFFFFFFFFLL ? 0xFFFFFFFFu : (uint32_t)us;
+                uint32_t qj = 0;   /* q_now of j, by the same definition */
+                for (int64_t jj = 0; jj < n; ++jj) {
+                    if (dev && dev[jj] != dev[j]) continue;
+                    int ib = (a[jj] < a[j]) || (a[jj] == a[j] && jj <= j);
+                    if (ib && c[jj] > a[j]) ++qj;
+                }
+                o[5 + k] = qj;
+            } else {
+                o[1 + k] = 0;
+                o[5 + k] = 0;
+            }
+        }
+    }
+}
+
 int oracle_max_threads(void)
 {
 #ifdef _OPENMP

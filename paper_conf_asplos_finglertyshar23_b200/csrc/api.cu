@@ -696,6 +696,26 @@ int lake_linnos_infer_host(const void *h_in, uint32_t flags, int64_t n, int32_t 
   return cuda_status(e);
 }
 
+size_t lake_linnos_capture_workspace_bytes(int64_t n) {
+  if (n < 0 || n > (int64_t)INT32_MAX) return 0;
+  return capture_workspace_bytes(n > 0 ? n : 1);
+}
+
+int lake_linnos_capture(const int64_t *arrival_ns, const int64_t *complete_ns,
+                        const int32_t *device, int64_t n, lake_io_raw_t *raw_out,
+                        void *workspace, size_t ws_bytes, void *stream) {
+  if (n < 0 || n > (int64_t)INT32_MAX) return LAKE_ERR_INVAL;
+  if (n == 0) return LAKE_OK;
+  if (!arrival_ns || !complete_ns || !raw_out || !workspace) return LAKE_ERR_INVAL;
+  if ((reinterpret_cast<uintptr_t>(arrival_ns) | reinterpret_cast<uintptr_t>(complete_ns)) & 7)
+    return LAKE_ERR_INVAL;
+  if (reinterpret_cast<uintptr_t>(raw_out) & 3) return LAKE_ERR_INVAL;
+  if (device && (reinterpret_cast<uintptr_t>(device) & 3)) return LAKE_ERR_INVAL;
+  return cuda_status(launch_capture(arrival_ns, complete_ns, device, n,
+                                    reinterpret_cast<uint32_t *>(raw_out), workspace, ws_bytes,
+                                    static_cast<cudaStream_t>(stream)));
+}
+
 uint64_t lake_linnos_launch_count(void) { return g_launches.load(); }
 void lake_linnos_reset_launch_count(void) { g_launches.store(0); }
 

@@ -90,6 +90,11 @@ struct GroupView {
 GroupView group_view(void *ws, int64_t n);
 size_t tc_smem_bytes(int nh_layout);
 
+// GPU feature capture (capture.cu)
+size_t capture_workspace_bytes(int64_t n);
+cudaError_t launch_capture(const int64_t *a, const int64_t *c, const int32_t *dev, int64_t n,
+                           uint32_t *raw, void *ws, size_t ws_bytes, cudaStream_t s);
+
 void count_launch(int k = 1);
 
 }  // namespace lake

@@ -37,6 +37,7 @@ EXPORTS = (
     "lake_linnos_multi_grouped", "lake_linnos_multi_status", "lake_linnos_host_staging_bytes",
     "lake_linnos_infer_host", "lake_linnos_launch_count", "lake_linnos_reset_launch_count",
     "lake_linnos_profile_enable", "lake_linnos_profile_read", "lake_linnos_strerror",
+    "lake_linnos_capture_workspace_bytes", "lake_linnos_capture",
 )
 
 
@@ -77,6 +78,8 @@ def lib():
             "lake_linnos_profile_enable": (ctypes.c_int, [ctypes.c_int]),
             "lake_linnos_profile_read": (ctypes.c_int, [P, P]),
             "lake_linnos_strerror": (ctypes.c_char_p, [ctypes.c_int]),
+            "lake_linnos_capture_workspace_bytes": (SZ, [I64]),
+            "lake_linnos_capture": (ctypes.c_int, [P, P, P, I64, P, P, SZ, P]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -203,3 +206,14 @@ def profile_read():
     _check(lib().lake_linnos_profile_read(ctypes.addressof(ms), ctypes.addressof(n)),
            "profile_read")
     return ms.value, n.value
+
+
+def capture_workspace_bytes(n: int) -> int:
+    return int(lib().lake_linnos_capture_workspace_bytes(n))
+
+
+def capture(arrival_ns, complete_ns, device, n: int, raw_out, workspace, ws_bytes: int,
+            stream=None) -> None:
+    _check(lib().lake_linnos_capture(_ptr(arrival_ns), _ptr(complete_ns), _ptr(device), n,
+                                     _ptr(raw_out), _ptr(workspace), ws_bytes, _stream(stream)),
+           "capture")

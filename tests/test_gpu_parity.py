@@ -308,3 +308,74 @@ def test_infer_host_pipelined_multi_equals_device(many_models):
     dlg, ddec, _ = run_multi(raw, ids, lake.LAKE_IN_RAW | lake.LAKE_PREC_F16)
     assert np.array_equal(dec, ddec)
     assert np.array_equal(lg.view(np.uint32), dlg.view(np.uint32))
+
+
+# ------------------------------------------------------------------------- feature capture
+def _gpu_capture(a, c, d):
+    import torch
+    n = a.shape[0]
+    ta = cuda(np.ascontiguousarray(a, np.int64))
+    tc_ = cuda(np.ascontiguousarray(c, np.int64))
+    td = cuda(np.ascontiguousarray(d, np.int32)) if d is not None else None
+    out = torch.full((n, 9), -1, dtype=torch.int32, device="cuda:0")
+    wsb = lake.capture_workspace_bytes(n)
+    ws = torch.empty(wsb, dtype=torch.uint8, device="cuda:0")
+    lake.capture(ta, tc_, td, n, out, ws, wsb)
+    torch.cuda.synchronize()
+    return out.cpu().numpy().view(np.uint32)
+
+
+def test_capture_hand_worked():
+    from conftest import read_golden
+    rows = read_golden("capture_example.txt")
+    d = np.array([int(r[1].split()[0]) for r in rows], np.int32)
+    a = np.array([int(r[1].split()[1]) for r in rows], np.int64)
+    c = np.array([int(r[1].split()[2]) for r in rows], np.int64)
+    exp = np.array([[int(v) for v in r[2].split()] for r in rows], np.uint32)
+    assert np.array_equal(_gpu_capture(a, c, d), exp)
+
+
+def _interleaved_trace(n, ndev, seed, quantum_ns=1):
+    rng = np.random.default_rng(seed)
+    parts_a, parts_c, parts_d = [], [], []
+    for dv in range(ndev):
+        tr = inputs.device_trace(inputs.PROFILE_ORDER[dv % 3], n // ndev, seed + dv, 3.0)
+        parts_a.append(tr["arrival_ns"] // quantum_ns * quantum_ns)
+        parts_c.append(np.maximum(tr["complete_ns"] // quantum_ns * quantum_ns,
+                                  parts_a[-1] + 1))
+        parts_d.append(np.full(n // ndev, dv, np.int32))
+    a, c, d = map(np.concatenate, (parts_a, parts_c, parts_d))
+    p = np.lexsort((rng.random(a.size), a))  # interleave by arrival, ties shuffled
+    return a[p], c[p], d[p]
+
+
+@pytest.mark.parametrize("quantum", [1, 1000])  # 1000 ns quanta: many exact ties
+def test_capture_equals_oracle(quantum):
+    a, c, d = _interleaved_trace(12000, 4, seed=70, quantum_ns=quantum)
+    assert np.array_equal(_gpu_capture(a, c, d), oracle.capture(a, c, d))
+
+
+def test_capture_full_size_sampled():
+    a, c, d = _interleaved_trace(1 << 20, 8, seed=80)
+    got = _gpu_capture(a, c, d)
+    rows = np.unique(np.concatenate([np.random.default_rng(2).choice(a.size, 300, replace=False),
+                                     np.arange(a.size - 5, a.size)]))
+    assert np.array_equal(got[rows], oracle.capture_rows(a, c, d, rows))
+
+
+def test_capture_then_infer_pipeline():
+    # NEXT-1 end to end on the device: trace -> capture -> per-model scoring
+    import torch
+    a, c, d = _interleaved_trace(9000, 3, seed=90)
+    models = {m: (2, inputs.weights(2, 300 + m)) for m in range(3)}
+    for m, (arch, blob) in models.items():
+        lake.load_weights(300 + m, arch, blob, 0)
+    raw_gpu = _gpu_capture(a, c, d)
+    ids = (300 + d).astype(np.int32)
+    lg, dec, _ = run_multi(raw_gpu, ids, lake.LAKE_IN_RAW | lake.LAKE_PREC_FP32)
+    raw_ref = oracle.capture(a, c, d)
+    rlg, rdec = oracle.infer_multi_raw({300 + m: v for m, v in models.items()}, raw_ref, ids)
+    assert np.array_equal(dec, rdec)
+    assert np.array_equal(lg.view(np.uint32), rlg.view(np.uint32))
+    for m in models:
+        lake.unload(300 + m, 0)
