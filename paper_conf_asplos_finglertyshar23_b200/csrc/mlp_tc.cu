@@ -69,8 +69,15 @@ namespace {
 #ifndef LAKE_EPI_PER_Q
 #define LAKE_EPI_PER_Q 2
 #endif
-constexpr uint32_t kEpiPerQ = LAKE_EPI_PER_Q;      // epilogue warps per TMEM lane quadrant
-constexpr uint32_t kEpiWarps = 4 * kEpiPerQ;       // 16
+constexpr uint32_t kEpiPerQ = LAKE_EPI_PER_Q;      // epilogue warps per group and quadrant
+// Epilogue groups: with 2, one group converts the H-producing layers (0..nh-2) and the
+// other the last layer (-> logits), so tile t's logits overlap tile t+1's first epilogues.
+#ifndef LAKE_EPI_GROUPS
+#define LAKE_EPI_GROUPS 2
+#endif
+constexpr uint32_t kEpiGroups = LAKE_EPI_GROUPS;
+constexpr uint32_t kGroupWarps = 4 * kEpiPerQ;     // warps per epilogue group
+constexpr uint32_t kEpiWarps = kEpiGroups * kGroupWarps;
 #ifndef LAKE_CHUNKS
 #define LAKE_CHUNKS 8
 #endif
@@ -88,14 +95,14 @@ constexpr uint32_t kHreadyCount = 2 * 4;               // one warp per quadrant,
 constexpr bool kInterleave = false;
 constexpr uint32_t kEpiCols = kChunkCols / kEpiPerQ;
 constexpr uint32_t kWarpChunks = kChunks;
-constexpr uint32_t kHreadyCount = 2 * kEpiWarps;
+constexpr uint32_t kHreadyCount = 2 * kGroupWarps;     // the H group's warps, both CTAs
 #endif
 constexpr uint32_t kKStepsPerChunk = kChunkCols / 16;
 constexpr int kThreads = 32 * (3 + kEpiWarps + 1);  // digitisers(2) + loader + epi + MMA
 constexpr uint32_t kHBytes = 128 * kHidden * 2;   // 64 KB
 constexpr uint32_t kXBytes = 128 * kTcK0 * 2;     // 8 KB
 constexpr uint32_t kLboR128 = 128 * 16;           // K-direction core stride, 128-row operand
-constexpr uint32_t kPrmFloats = kMaxHiddenLayers * kHidden + 2 * kHidden + 4;  // biases|Wout|bout
+constexpr uint32_t kPrmFloats = kHidden + 2 * kHidden + 4;  // last-layer bias | W_out | b_out
 constexpr uint32_t kPrm2Words = (kMaxHiddenLayers - 1) * kHidden / 2;  // packed bias pairs
 constexpr uint32_t kRedBytes = (kEpiPerQ - 1) * 128 * 2 * 4;  // output-layer partial sums
 
@@ -117,8 +124,8 @@ __host__ __device__ constexpr Layout tc_layout(int nh_layout) {
 
 // barrier slots (8 bytes each) inside the barrier block
 enum : uint32_t {
-  B_WLOAD = 0, B_WREADY = 1, B_XFULL = 2, B_XEMPTY = 4, B_DFULL = 6, B_TEMPTY = 8,
-  B_HREADY = 10, B_WFREE = 10 + kChunks, B_COUNT = 11 + kChunks
+  B_WLOAD = 0, B_WREADY = 1, B_XFULL = 2, B_XEMPTY = 4, B_DFULL = 6, B_DFULLX = 8,
+  B_TEMPTY = 10, B_HREADY = 12, B_WFREE = 12 + kChunks, B_COUNT = 13 + kChunks
 };
 constexpr uint32_t kTmemSlot = B_COUNT * 8;  // u32 TMEM base address
 
@@ -244,8 +251,9 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
     for (int i = 0; i < 2; ++i) {
       ptx::mbar_init(bar(B_XFULL + i), 2);       // one arrive per CTA digitiser group
       ptx::mbar_init(bar(B_XEMPTY + i), 1);      // tcgen05.commit (multicast)
-      ptx::mbar_init(bar(B_DFULL + i), 1);       // tcgen05.commit (multicast)
-      ptx::mbar_init(bar(B_TEMPTY + i), 2 * kEpiWarps);  // every epilogue warp, both CTAs
+      ptx::mbar_init(bar(B_DFULL + i), 1);       // tcgen05.commit (multicast): H layers
+      ptx::mbar_init(bar(B_DFULLX + i), 1);      // tcgen05.commit (multicast): last layer
+      ptx::mbar_init(bar(B_TEMPTY + i), 2 * kGroupWarps);  // the draining group, both CTAs
     }
     for (uint32_t i = 0; i < kChunks; ++i) ptx::mbar_init(bar(B_HREADY + i), kHreadyCount);
     ptx::mbar_init(bar(B_WFREE), 1);             // tcgen05.commit (multicast)
@@ -344,7 +352,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           for (uint32_t s = 0; s < kTcK0 / 16; ++s)
             ptx::mma_f16_cg2(d, xd + s * kStep, w0desc + s * kStep, idesc, s);
           ptx::mma_commit_cg2(bar(B_XEMPTY + xb), 0x3);
-          ptx::mma_commit_cg2(bar(B_DFULL + b), 0x3);
+          ptx::mma_commit_cg2(bar((kEpiGroups == 2 && nh == 1 ? B_DFULLX : B_DFULL) + b), 0x3);
           LAKE_TEV(T_COMMIT, it, 0, 0);
           ++g;
         }
@@ -377,7 +385,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
 #endif
             LAKE_TEV(T_ISSUED, it, l, kc);
           }
-          ptx::mma_commit_cg2(bar(B_DFULL + b), 0x3);
+          ptx::mma_commit_cg2(bar((kEpiGroups == 2 && l + 1 == nh ? B_DFULLX : B_DFULL) + b), 0x3);
           LAKE_TEV(T_COMMIT, it, l, 0);
           ++g;
         }
@@ -444,20 +452,24 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
     }
   } else if (warp >= kWarpEpi && warp < kWarpEpi + kEpiWarps) {
     // ================= epilogue =================
-    constexpr uint32_t NE = kEpiWarps * 32;           // epilogue threads
+    constexpr uint32_t NG = kGroupWarps * 32;         // threads per epilogue group
     constexpr int W = kEpiCols;
-    const uint32_t et = threadIdx.x - kWarpEpi * 32;  // 0..NE-1
+    const uint32_t gy = (warp - kWarpEpi) / kGroupWarps;  // 0: H layers (or all), 1: last layer
+    const uint32_t lw = (warp - kWarpEpi) % kGroupWarps;
+    const uint32_t et = lw * 32 + lane;                   // thread index within the group
     const uint32_t q = warp & 3;                      // TMEM lane quadrant this warp may access
-    const uint32_t hh = (warp - kWarpEpi) >> 2;       // which W-column slice of each chunk
+    const uint32_t hh = lw >> 2;                      // which W-column slice of each chunk
     const uint32_t row = q * 32 + lane;     // row within this CTA's 128
+    const bool do_h = kEpiGroups == 1 || gy == 0;     // converts H-producing layers
+    const bool do_last = kEpiGroups == 1 || gy == 1;  // converts the last layer
     const uint32_t hready_leader0 = ptx::mapa(bar(B_HREADY), 0);
     const uint32_t tempty_leader0 = ptx::mapa(bar(B_TEMPTY), 0);
     const uint32_t hrow = sbase + L.h + row * 16;
-    float *prm = reinterpret_cast<float *>(smem + L.prm);
+    float *prm = reinterpret_cast<float *>(smem + L.prm);    // last bias | W_out | b_out
     uint32_t *prm2 = reinterpret_cast<uint32_t *>(smem + L.prm + kPrmFloats * 4);
     float *red = reinterpret_cast<float *>(smem + L.red);
     const DevModel *cur = nullptr;
-    uint32_t g = 0, d_phase = 0;  // d_phase: bit b
+    uint32_t g = 0, d_phase = 0, dx_phase = 0;  // phase bits per accumulator buffer
     int64_t it = 0;
     TileInfo nxt;
     if (t_begin < t_end) nxt = tile_info<PREC>(ts, t_begin);
@@ -470,24 +482,35 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
 #endif
       const int nh = ti.nh;
       if (ti.model != cur) {
-        // stage this model's fp32 biases | W_out | b_out (contiguous in its FP32 image)
-        const uint32_t nf4 = (nh * kHidden + 2 * kHidden + 4) / 4;
-        ptx::named_bar_sync(2, NE);
-        const float4 *src = reinterpret_cast<const float4 *>(ti.model->b[0]);
-        for (uint32_t i = et; i < nf4; i += NE) reinterpret_cast<float4 *>(prm)[i] = __ldg(src + i);
-        // hidden-layer biases feeding an MMA, as packed operand-type pairs
-        for (uint32_t i = et; i < (uint32_t)(nh - 1) * kHidden / 2; i += NE) {
-          const float2 bf = __ldg(reinterpret_cast<const float2 *>(ti.model->b[0]) + i);
-          prm2[i] = PREC == 0 ? ptx::pack_f16(bf.x, bf.y) : ptx::pack_bf16(bf.x, bf.y);
+        // stage this model's epilogue parameters (each group the ones it uses): packed
+        // operand-type bias pairs of the H layers, fp32 last-layer bias | W_out | b_out
+        ptx::named_bar_sync(2 + gy, NG);
+        if (do_h) {
+          for (uint32_t i = et; i < (uint32_t)(nh - 1) * kHidden / 2; i += NG) {
+            const float2 bf = __ldg(reinterpret_cast<const float2 *>(ti.model->b[0]) + i);
+            prm2[i] = PREC == 0 ? ptx::pack_f16(bf.x, bf.y) : ptx::pack_bf16(bf.x, bf.y);
+          }
         }
-        ptx::named_bar_sync(2, NE);
+        if (do_last) {
+          const float4 *src = reinterpret_cast<const float4 *>(ti.model->b[nh - 1]);
+          for (uint32_t i = et; i < kPrmFloats / 4; i += NG)
+            reinterpret_cast<float4 *>(prm)[i] = __ldg(src + i);
+        }
+        ptx::named_bar_sync(2 + gy, NG);
         cur = ti.model;
       }
-      const float *wo = prm + nh * kHidden;
-      for (int l = 0; l < nh; ++l) {
+      const float *wo = prm + kHidden;
+      for (int l = 0; l < nh; ++l, ++g) {
+        const bool last = (l + 1 == nh);
+        if (!(last ? do_last : do_h)) continue;
         const uint32_t b = g & 1;
-        ptx::mbar_wait(bar(B_DFULL + b), (d_phase >> b) & 1);
-        d_phase ^= (1u << b);
+        if (kEpiGroups == 2 && last) {
+          ptx::mbar_wait(bar(B_DFULLX + b), (dx_phase >> b) & 1);
+          dx_phase ^= (1u << b);
+        } else {
+          ptx::mbar_wait(bar(B_DFULL + b), (d_phase >> b) & 1);
+          d_phase ^= (1u << b);
+        }
         LAKE_TEV(T_DFULL, it, l, warp);
         ptx::tc_fence_after();
         const uint32_t tbase = tmem + ((q * 32) << 16) + b * 256;
@@ -496,7 +519,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         auto col_of = [&](uint32_t j) {
           return kInterleave ? chunk_of(j) * kChunkCols : j * kChunkCols + hh * W;
         };
-        const float *bl = prm + l * kHidden;
+        const float *bl = prm;  // last-layer bias
 #ifdef LAKE_NO_EPI_PREFETCH
         constexpr bool kPrefetch = false;
 #else
@@ -505,7 +528,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         uint32_t ra[W], rb[W];  // rb unused (eliminated) without prefetch
         ptx::tmem_ld_cols<W>(tbase + col_of(0), ra);
         ptx::tmem_ld_wait();
-        if (l + 1 < nh) {
+        if (!last) {
           // hidden layer feeding another MMA; with two register buffers the TMEM load of the
           // warp's next chunk is in flight while the current one is converted and stored
 #pragma unroll
@@ -563,7 +586,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
             rd[0] = p0;
             rd[1] = p1;
           }
-          ptx::named_bar_sync(3 + q, 32 * kEpiPerQ);
+          ptx::named_bar_sync(4 + q, 32 * kEpiPerQ);
           if (hh == 0) {
 #pragma unroll
             for (uint32_t j = 0; j + 1 < kEpiPerQ; ++j) {
@@ -571,9 +594,9 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
               p1 += red[(j * 128 + row) * 2 + 1];
             }
           }
-          // NN (one layer per tile): nothing else orders the next tile's partial writes
-          // after this read, so close the exchange explicitly
-          if (nh == 1) ptx::named_bar_sync(3 + q, 32 * kEpiPerQ);
+          // close the exchange before the partial sums are overwritten by the next tile
+          // (single group: only NN lacks a later ordering point)
+          if (kEpiGroups == 2 || nh == 1) ptx::named_bar_sync(4 + q, 32 * kEpiPerQ);
           if (hh == 0) {
             const float l0 = p0 + wo[2 * kHidden + 0];
             const float l1 = p1 + wo[2 * kHidden + 1];
@@ -594,7 +617,6 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         __syncwarp();
         if (lane == 0) ptx::mbar_arrive_cluster(tempty_leader0 + b * 8);
         LAKE_TEV(T_LAYER_END, it, l, warp);
-        ++g;
       }
     }
   }
