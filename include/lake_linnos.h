@@ -99,11 +99,19 @@ enum lake_flags {
     LAKE_PREC_F16   = 0x10, /* tcgen05 tensor cores, fp16 operands, fp32 accumulation     */
     LAKE_PREC_BF16  = 0x20, /* tcgen05 tensor cores, bf16 operands, fp32 accumulation     */
     LAKE_PREC_TF32  = 0x30, /* reserved: returns LAKE_ERR_UNSUPPORTED (SMEM)   */
-    LAKE_PREC_AUTO  = 0x70, /* FP32 below LAKE_AUTO_TC_MIN_N I/Os per call, else F16      */
+    LAKE_PREC_AUTO  = 0x70, /* FP32 below the model's AUTO threshold, else F16 (below)   */
     LAKE_IN_MASK    = 0x01,
     LAKE_PREC_MASK  = 0x70
 };
-#define LAKE_AUTO_TC_MIN_N 2048
+/* LAKE_PREC_AUTO (the paper's profitability policy, §4.2 P:583-603 and
+ * Fig. 3, restricted to GPU paths since there is no CPU fallback): a call with n
+ * I/Os takes the bit-exact FP32 path when n < threshold(arch), else the fp16 tensor-core
+ * path. Defaults come from the measured C2 curves (profiles/*_sweep_c2.jsonl): the tensor
+ * path is chosen where it is at least 20% faster end to end than FP32 — for NN never
+ * within the 1..4096 sweep (threshold 8192), for NN+1 and NN+2 from one I/O on. */
+#define LAKE_AUTO_TC_MIN_N_NN  8192
+#define LAKE_AUTO_TC_MIN_N_NN1 1
+#define LAKE_AUTO_TC_MIN_N_NN2 1
 
 #define LAKE_MAX_MODELS 1024   /* model_id range: [0, LAKE_MAX_MODELS) per device */
 
@@ -127,6 +135,11 @@ int lake_linnos_unload(int32_t model_id, int32_t device);
 
 /* Architecture of a loaded model through *arch_out; LAKE_ERR_NOMODEL if not loaded. */
 int lake_linnos_model_arch(int32_t model_id, int32_t device, int32_t *arch_out);
+
+/* Read / override the AUTO threshold of an architecture (process-wide). Setting returns
+ * LAKE_ERR_INVAL for an unknown arch or n_min < 0. */
+int lake_linnos_auto_threshold(int32_t arch, int64_t *n_min_out);
+int lake_linnos_set_auto_threshold(int32_t arch, int64_t n_min);
 
 /* Digitisation kernel (integer, bit-exact). raw: device lake_io_raw_t[n];
  * digits: device uint8_t[n][32], layout above. n == 0 is a no-op. */

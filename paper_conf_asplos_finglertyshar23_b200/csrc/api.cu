@@ -208,7 +208,20 @@ int current_table(int *device, const DevModel **table, int *any) {
   return LAKE_OK;
 }
 
-int check_flags(uint32_t flags, int64_t n, int *in_kind, int *prec) {
+std::atomic<int64_t> g_auto_min[3] = {{LAKE_AUTO_TC_MIN_N_NN}, {LAKE_AUTO_TC_MIN_N_NN1},
+                                      {LAKE_AUTO_TC_MIN_N_NN2}};
+
+// arch < 0: unknown here (multi-model / host path before lookup) -> most conservative
+int64_t auto_min(int32_t arch) {
+  if (arch < 0 || arch > 2) {
+    int64_t m = 0;
+    for (int a = 0; a < 3; ++a) m = g_auto_min[a].load() > m ? g_auto_min[a].load() : m;
+    return m;
+  }
+  return g_auto_min[arch].load();
+}
+
+int check_flags(uint32_t flags, int64_t n, int *in_kind, int *prec, int32_t arch = -1) {
   if (flags & ~(uint32_t)(LAKE_IN_MASK | LAKE_PREC_MASK)) return LAKE_ERR_INVAL;
   *in_kind = (int)(flags & LAKE_IN_MASK);
   const uint32_t p = flags & LAKE_PREC_MASK;
@@ -217,7 +230,7 @@ int check_flags(uint32_t flags, int64_t n, int *in_kind, int *prec) {
     case LAKE_PREC_F16: *prec = 0; break;
     case LAKE_PREC_BF16: *prec = 1; break;
     case LAKE_PREC_TF32: return LAKE_ERR_UNSUPPORTED;
-    case LAKE_PREC_AUTO: *prec = (n >= LAKE_AUTO_TC_MIN_N) ? 0 : -1; break;
+    case LAKE_PREC_AUTO: *prec = (n >= auto_min(arch)) ? 0 : -1; break;
     default: return LAKE_ERR_INVAL;
   }
   return LAKE_OK;
@@ -417,6 +430,7 @@ int lake_linnos_infer(const void *in, uint32_t flags, int64_t n, int32_t model_i
   DevModel m;
   rc = current_model(model_id, &device, &m, nullptr);
   if (rc != LAKE_OK) return rc;
+  if ((flags & LAKE_PREC_MASK) == LAKE_PREC_AUTO) check_flags(flags, n, &in_kind, &prec, m.arch);
   TileSched ts;
   std::memset(&ts, 0, sizeof(ts));
   const int rows = prec < 0 ? kF32TileM : kTcTileRows;
@@ -425,6 +439,18 @@ int lake_linnos_infer(const void *in, uint32_t flags, int64_t n, int32_t model_i
   ts.model = m;
   return launch_main(in, in_kind, prec, ts, m.nh, decisions, logits,
                      static_cast<cudaStream_t>(stream), device);
+}
+
+int lake_linnos_auto_threshold(int32_t arch, int64_t *n_min_out) {
+  if (arch < 0 || arch > 2 || !n_min_out) return LAKE_ERR_INVAL;
+  *n_min_out = g_auto_min[arch].load();
+  return LAKE_OK;
+}
+
+int lake_linnos_set_auto_threshold(int32_t arch, int64_t n_min) {
+  if (arch < 0 || arch > 2 || n_min < 0) return LAKE_ERR_INVAL;
+  g_auto_min[arch].store(n_min);
+  return LAKE_OK;
 }
 
 size_t lake_linnos_workspace_bytes(int64_t n) {
@@ -592,16 +618,20 @@ int lake_linnos_infer_host(const void *h_in, uint32_t flags, int64_t n, int32_t 
   if (n == 0) return LAKE_OK;
   if (!h_in || !h_decisions || !d_staging) return LAKE_ERR_INVAL;
   if (staging_bytes < lake_linnos_host_staging_bytes(n, flags)) return LAKE_ERR_NOMEM;
-  // AUTO decides on the whole batch, not per chunk
-  if ((flags & LAKE_PREC_MASK) == LAKE_PREC_AUTO)
-    flags = (flags & ~(uint32_t)LAKE_PREC_MASK) | (prec < 0 ? LAKE_PREC_FP32 : LAKE_PREC_F16);
   int device;
   if (cudaGetDevice(&device) != cudaSuccess) return LAKE_ERR_CUDA;
   if (device < 0 || device >= kMaxDevices) return LAKE_ERR_INVAL;
+  int32_t arch = -1;
   if (!h_model_ids) {  // validate the single model once, before any copy
     DevModel m;
     rc = current_model(model_id, &device, &m, nullptr);
     if (rc != LAKE_OK) return rc;
+    arch = m.arch;
+  }
+  // AUTO decides on the whole batch, not per chunk
+  if ((flags & LAKE_PREC_MASK) == LAKE_PREC_AUTO) {
+    check_flags(flags, n, &in_kind, &prec, arch);
+    flags = (flags & ~(uint32_t)LAKE_PREC_MASK) | (prec < 0 ? LAKE_PREC_FP32 : LAKE_PREC_F16);
   }
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   const size_t in_b = in_kind == LAKE_IN_RAW ? 36 : 32;

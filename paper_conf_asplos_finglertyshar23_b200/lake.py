@@ -24,7 +24,7 @@ LAKE_IN_DIGITS, LAKE_IN_RAW = 0x00, 0x01
 LAKE_PREC_FP32, LAKE_PREC_F16, LAKE_PREC_BF16, LAKE_PREC_TF32, LAKE_PREC_AUTO = (
     0x00, 0x10, 0x20, 0x30, 0x70)
 LAKE_MAX_MODELS = 1024
-LAKE_AUTO_TC_MIN_N = 2048
+LAKE_AUTO_TC_MIN_N = {0: 8192, 1: 1, 2: 1}  # defaults (include/lake_linnos.h)
 
 PREC_FLAGS = {"fp32": LAKE_PREC_FP32, "f16": LAKE_PREC_F16, "bf16": LAKE_PREC_BF16,
               "tf32": LAKE_PREC_TF32, "auto": LAKE_PREC_AUTO}
@@ -38,6 +38,7 @@ EXPORTS = (
     "lake_linnos_infer_host", "lake_linnos_launch_count", "lake_linnos_reset_launch_count",
     "lake_linnos_profile_enable", "lake_linnos_profile_read", "lake_linnos_strerror",
     "lake_linnos_capture_workspace_bytes", "lake_linnos_capture",
+    "lake_linnos_auto_threshold", "lake_linnos_set_auto_threshold",
 )
 
 
@@ -80,6 +81,8 @@ def lib():
             "lake_linnos_strerror": (ctypes.c_char_p, [ctypes.c_int]),
             "lake_linnos_capture_workspace_bytes": (SZ, [I64]),
             "lake_linnos_capture": (ctypes.c_int, [P, P, P, I64, P, P, SZ, P]),
+            "lake_linnos_auto_threshold": (ctypes.c_int, [I32, P]),
+            "lake_linnos_set_auto_threshold": (ctypes.c_int, [I32, I64]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -217,3 +220,13 @@ def capture(arrival_ns, complete_ns, device, n: int, raw_out, workspace, ws_byte
     _check(lib().lake_linnos_capture(_ptr(arrival_ns), _ptr(complete_ns), _ptr(device), n,
                                      _ptr(raw_out), _ptr(workspace), ws_bytes, _stream(stream)),
            "capture")
+
+
+def auto_threshold(arch: int) -> int:
+    out = ctypes.c_int64(0)
+    _check(lib().lake_linnos_auto_threshold(arch, ctypes.addressof(out)), "auto_threshold")
+    return out.value
+
+
+def set_auto_threshold(arch: int, n_min: int) -> None:
+    _check(lib().lake_linnos_set_auto_threshold(arch, n_min), "set_auto_threshold")

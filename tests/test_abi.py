@@ -90,3 +90,14 @@ def test_product_never_touches_oracle(path):
     assert "oracle" not in src.replace("bit-exact with the\n// oracle", "").lower() or \
         "import oracle" not in src
     assert "import oracle" not in src and "liblake_oracle" not in src
+
+
+def test_auto_thresholds_roundtrip():
+    assert [lake.auto_threshold(a) for a in range(3)] == [lake.LAKE_AUTO_TC_MIN_N[a] for a in range(3)]
+    lake.set_auto_threshold(1, 777)
+    assert lake.auto_threshold(1) == 777
+    lake.set_auto_threshold(1, lake.LAKE_AUTO_TC_MIN_N[1])
+    with pytest.raises(lake.LakeError):
+        lake.set_auto_threshold(5, 1)
+    with pytest.raises(lake.LakeError):
+        lake.set_auto_threshold(0, -1)

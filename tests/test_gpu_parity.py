@@ -379,3 +379,21 @@ def test_capture_then_infer_pipeline():
     assert np.array_equal(lg.view(np.uint32), rlg.view(np.uint32))
     for m in models:
         lake.unload(300 + m, 0)
+
+
+def test_auto_policy_routes_by_arch_and_size():
+    # NN below its threshold -> bit-exact FP32; NN+2 -> tensor-core path
+    raw = _trace(300, seed=61)
+    lg, dec = run_infer(10, raw, lake.LAKE_IN_RAW | lake.LAKE_PREC_AUTO)
+    rlg, rdec = oracle.infer_raw(0, inputs.weights(0, 10), raw, nthreads=0)
+    assert np.array_equal(lg.view(np.uint32), rlg.view(np.uint32))
+    lg2, _ = run_infer(12, raw, lake.LAKE_IN_RAW | lake.LAKE_PREC_AUTO)
+    tlg, _ = run_infer(12, raw, lake.LAKE_IN_RAW | lake.LAKE_PREC_F16)
+    assert np.array_equal(lg2.view(np.uint32), tlg.view(np.uint32))
+    lake.set_auto_threshold(2, 10**9)  # force FP32 for NN+2
+    try:
+        lg3, _ = run_infer(12, raw, lake.LAKE_IN_RAW | lake.LAKE_PREC_AUTO)
+        r3, _ = oracle.infer_raw(2, inputs.weights(2, 12), raw, nthreads=0)
+        assert np.array_equal(lg3.view(np.uint32), r3.view(np.uint32))
+    finally:
+        lake.set_auto_threshold(2, lake.LAKE_AUTO_TC_MIN_N[2])
