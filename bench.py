@@ -420,6 +420,7 @@ def run_sweep(args):
         for prec in ("fp32", "f16", "bf16"):
             flags = lake.LAKE_IN_RAW | lake.PREC_FLAGS[prec]
             cross = None
+            scross = None
             for b in sizes:
                 raw = np.ascontiguousarray(raw_all[:b])
                 h_in = torch.from_numpy(raw.view(np.int32)).pin_memory()
@@ -458,9 +459,25 @@ def run_sweep(args):
                 row = dict(arch=ARCH_NAME[arch], prec=prec, batch=b, e2e_us_median=round(med, 2),
                            e2e_us_p99=round(float(np.percentile(ts, 99)), 2),
                            device_us=round(dev_us, 2), cpu_1thread_us=round(cpu_us, 2))
+                if prec == "fp32" and b <= lake.LAKE_SERVER_MAX_BATCH:
+                    # NEXT-2: persistent resident-weights server (doorbell, no launch/copies)
+                    sdec = np.zeros(b, np.uint8)
+                    with lake.Server(40 + arch) as srv:
+                        for _ in range(warm):
+                            srv.infer(raw, b, sdec)
+                        st = []
+                        for _ in range(reps):
+                            t0 = time.perf_counter()
+                            srv.infer(raw, b, sdec)
+                            st.append((time.perf_counter() - t0) * 1e6)
+                    row["server_us_median"] = round(float(np.median(st)), 2)
+                    row["server_us_p99"] = round(float(np.percentile(st, 99)), 2)
+                    if scross is None and row["server_us_median"] < cpu_us:
+                        scross = b
                 out.append(row)
                 log(json.dumps(row))
-            out.append(dict(arch=ARCH_NAME[arch], prec=prec, crossover_batch=cross))
+            out.append(dict(arch=ARCH_NAME[arch], prec=prec, crossover_batch=cross,
+                            **({"server_crossover_batch": scross} if prec == "fp32" else {})))
             log(json.dumps(out[-1]))
         lake.unload(40 + arch, 0)
     path = args.sweep_out or os.path.join(ROOT, "gpurun_out", "sweep.jsonl")

@@ -125,8 +125,10 @@ size_t lake_linnos_blob_floats(int32_t arch);
  *     W0[256][31] b0[256]  (W1[256][256] b1[256])  (W2[256][256] b2[256])  Wout[2][256] bout[2]
  * n_floats must equal lake_linnos_blob_floats(arch), else LAKE_ERR_INVAL.
  * device: CUDA ordinal the model is loaded on (the current device is restored on return).
- * Replaces any model already loaded under (model_id, device). Synchronous. The library
- * deep-copies the blob into device-resident FP32 / fp16 / bf16 images it owns. */
+ * Replaces any model already loaded under (model_id, device). Synchronous with respect to
+ * the host (no device-wide synchronisation: the caller must not load/unload a model that an
+ * in-flight infer uses). The library deep-copies the blob into device-resident FP32 / fp16 /
+ * bf16 images it owns. */
 int lake_linnos_load_weights(int32_t model_id, int32_t arch, const float *blob,
                              size_t n_floats, int32_t device);
 
@@ -217,6 +219,26 @@ size_t lake_linnos_capture_workspace_bytes(int64_t n);
 int lake_linnos_capture(const int64_t *arrival_ns, const int64_t *complete_ns,
                         const int32_t *device, int64_t n, lake_io_raw_t *raw_out,
                         void *workspace, size_t ws_bytes, void *stream);
+
+/* Persistent resident-weights server: the latency path for small
+ * batches, against the paper's profitability problem (§4.2; Fig. 8).
+ * _server_start launches one kernel that stays resident on an 8-CTA cluster (8 SMs) with a
+ * slice of the model's FP32 weights in each CTA's shared memory, and a mailbox in mapped
+ * pinned host memory. _server_infer copies up to LAKE_SERVER_MAX_BATCH raw records (HOST
+ * pointer) into the mailbox, rings the doorbell (a sequence number the kernel polls with
+ * system-scope acquire loads), and spins until the kernel has written the decisions (and
+ * logits if non-NULL, HOST pointers) back into the mailbox: no launch, no memcpy, no stream
+ * sync per batch. Arithmetic = the FP32 path (bit-exact with the oracle). Calls on one
+ * server must not overlap (one batch in flight). The server keeps its own copy of the
+ * weights: unloading the model afterwards is safe. _server_stop ends the kernel.
+ * Errors: LAKE_ERR_INVAL (n < 0 or > LAKE_SERVER_MAX_BATCH, NULL), LAKE_ERR_NOMODEL,
+ * LAKE_ERR_CUDA (the kernel died or never answered). */
+#define LAKE_SERVER_MAX_BATCH 64
+typedef struct lake_server lake_server_t;
+int lake_linnos_server_start(int32_t model_id, lake_server_t **server_out);
+int lake_linnos_server_infer(lake_server_t *server, const lake_io_raw_t *h_raw, int32_t n,
+                             uint8_t *h_decisions, float *h_logits);
+int lake_linnos_server_stop(lake_server_t *server);
 
 /* Number of kernels this library launched on the current device since the last reset
  * (host-side counter; used by the bench to report gpu_launches). */

@@ -37,6 +37,10 @@ struct DeviceState {
   DevModel host[LAKE_MAX_MODELS];
   ModelBufs bufs[LAKE_MAX_MODELS];
   DevModel *table = nullptr;  // device copy
+  // cudaFree synchronises the device, which never completes while a persistent server
+  // kernel runs: replaced buffers wait here until no server is active on the device
+  std::vector<ModelBufs> graveyard;
+  int servers = 0;
 };
 
 std::mutex g_mu;
@@ -160,6 +164,23 @@ void free_bufs(ModelBufs &b) {
   if (b.fp32) cudaFree(b.fp32);
   if (b.tc) cudaFree(b.tc);
   b.fp32 = b.tc = nullptr;
+}
+
+// Release replaced model buffers now, or later if a persistent server is running.
+void retire_bufs(DeviceState *st, ModelBufs &b) {
+  if (!b.fp32 && !b.tc) return;
+  if (st->servers > 0) {
+    st->graveyard.push_back(b);
+    b.fp32 = b.tc = nullptr;
+  } else {
+    free_bufs(b);
+  }
+}
+
+void flush_graveyard(DeviceState *st) {
+  if (st->servers > 0) return;
+  for (auto &b : st->graveyard) free_bufs(b);
+  st->graveyard.clear();
 }
 
 int cuda_status(cudaError_t e) {
@@ -343,12 +364,12 @@ int lake_linnos_load_weights(int32_t model_id, int32_t arch, const float *blob, 
   ModelBufs nb;
   if (cudaMalloc(&nb.fp32, f_total * 4) != cudaSuccess) return LAKE_ERR_NOMEM;
   if (cudaMalloc(&nb.tc, img.size()) != cudaSuccess) {
-    free_bufs(nb);
+    retire_bufs(st, nb);
     return LAKE_ERR_NOMEM;
   }
   if (cudaMemcpy(nb.fp32, f.data(), f_total * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
       cudaMemcpy(nb.tc, img.data(), img.size(), cudaMemcpyHostToDevice) != cudaSuccess) {
-    free_bufs(nb);
+    retire_bufs(st, nb);
     return LAKE_ERR_CUDA;
   }
   DevModel m;
@@ -365,13 +386,14 @@ int lake_linnos_load_weights(int32_t model_id, int32_t arch, const float *blob, 
   }
   m.wout = fb + off_wout;
   m.bout = fb + off_bout;
-  // publish: device table entry, then host mirror; free the previous buffers
-  if (cudaDeviceSynchronize() != cudaSuccess ||
-      cudaMemcpy(st->table + model_id, &m, sizeof(m), cudaMemcpyHostToDevice) != cudaSuccess) {
-    free_bufs(nb);
+  // publish: device table entry, then host mirror; retire the previous buffers. (No
+  // device-wide sync: in-flight work on this model is excluded by the header's contract.)
+  if (cudaMemcpy(st->table + model_id, &m, sizeof(m), cudaMemcpyHostToDevice) != cudaSuccess) {
+    retire_bufs(st, nb);
     return LAKE_ERR_CUDA;
   }
-  free_bufs(st->bufs[model_id]);
+  retire_bufs(st, st->bufs[model_id]);
+  flush_graveyard(st);
   st->bufs[model_id] = nb;
   st->host[model_id] = m;
   return LAKE_OK;
@@ -388,10 +410,10 @@ int lake_linnos_unload(int32_t model_id, int32_t device) {
   DevModel m;
   std::memset(&m, 0, sizeof(m));
   m.arch = -1;
-  if (cudaDeviceSynchronize() != cudaSuccess ||
-      cudaMemcpy(st->table + model_id, &m, sizeof(m), cudaMemcpyHostToDevice) != cudaSuccess)
+  if (cudaMemcpy(st->table + model_id, &m, sizeof(m), cudaMemcpyHostToDevice) != cudaSuccess)
     return LAKE_ERR_CUDA;
-  free_bufs(st->bufs[model_id]);
+  retire_bufs(st, st->bufs[model_id]);
+  flush_graveyard(st);
   st->host[model_id] = m;
   return LAKE_OK;
 }
@@ -744,6 +766,45 @@ int lake_linnos_capture(const int64_t *arrival_ns, const int64_t *complete_ns,
   return cuda_status(launch_capture(arrival_ns, complete_ns, device, n,
                                     reinterpret_cast<uint32_t *>(raw_out), workspace, ws_bytes,
                                     static_cast<cudaStream_t>(stream)));
+}
+
+int lake_linnos_server_start(int32_t model_id, lake_server_t **server_out) {
+  if (!server_out) return LAKE_ERR_INVAL;
+  int device;
+  DevModel m;
+  int rc = current_model(model_id, &device, &m, nullptr);
+  if (rc != LAKE_OK) return rc;
+  Server *s = nullptr;
+  rc = server_start(m, device, &s);
+  if (rc != LAKE_OK) return rc;
+  {
+    std::lock_guard<std::mutex> lk(g_mu);
+    g_dev[device]->servers++;
+  }
+  *server_out = reinterpret_cast<lake_server_t *>(s);
+  return LAKE_OK;
+}
+
+int lake_linnos_server_infer(lake_server_t *server, const lake_io_raw_t *h_raw, int32_t n,
+                             uint8_t *h_decisions, float *h_logits) {
+  if (!server || n < 0 || n > LAKE_SERVER_MAX_BATCH) return LAKE_ERR_INVAL;
+  if (n == 0) return LAKE_OK;
+  if (!h_raw || !h_decisions) return LAKE_ERR_INVAL;
+  return server_infer(reinterpret_cast<Server *>(server), h_raw, n, h_decisions, h_logits);
+}
+
+int lake_linnos_server_stop(lake_server_t *server) {
+  if (!server) return LAKE_ERR_INVAL;
+  const int device = server_device(reinterpret_cast<Server *>(server));
+  const int rc = server_stop(reinterpret_cast<Server *>(server));
+  std::lock_guard<std::mutex> lk(g_mu);
+  DeviceState *st = g_dev[device];
+  if (st && st->servers > 0) {
+    st->servers--;
+    DeviceGuard dg(device);
+    flush_graveyard(st);
+  }
+  return rc;
 }
 
 uint64_t lake_linnos_launch_count(void) { return g_launches.load(); }

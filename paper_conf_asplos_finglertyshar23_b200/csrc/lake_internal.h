@@ -95,6 +95,14 @@ size_t capture_workspace_bytes(int64_t n);
 cudaError_t launch_capture(const int64_t *a, const int64_t *c, const int32_t *dev, int64_t n,
                            uint32_t *raw, void *ws, size_t ws_bytes, cudaStream_t s);
 
+// persistent doorbell server (server.cu)
+struct Server;
+int server_start(const DevModel &m, int device, Server **out);
+int server_infer(Server *s, const lake_io_raw_t *raw, int32_t n, uint8_t *dec, float *logits);
+int server_stop(Server *s);
+size_t server_smem_bytes();
+int server_device(const Server *s);
+
 void count_launch(int k = 1);
 
 }  // namespace lake

@@ -24,6 +24,7 @@ LAKE_IN_DIGITS, LAKE_IN_RAW = 0x00, 0x01
 LAKE_PREC_FP32, LAKE_PREC_F16, LAKE_PREC_BF16, LAKE_PREC_TF32, LAKE_PREC_AUTO = (
     0x00, 0x10, 0x20, 0x30, 0x70)
 LAKE_MAX_MODELS = 1024
+LAKE_SERVER_MAX_BATCH = 64
 LAKE_AUTO_TC_MIN_N = {0: 8192, 1: 1, 2: 1}  # defaults (include/lake_linnos.h)
 
 PREC_FLAGS = {"fp32": LAKE_PREC_FP32, "f16": LAKE_PREC_F16, "bf16": LAKE_PREC_BF16,
@@ -39,6 +40,7 @@ EXPORTS = (
     "lake_linnos_profile_enable", "lake_linnos_profile_read", "lake_linnos_strerror",
     "lake_linnos_capture_workspace_bytes", "lake_linnos_capture",
     "lake_linnos_auto_threshold", "lake_linnos_set_auto_threshold",
+    "lake_linnos_server_start", "lake_linnos_server_infer", "lake_linnos_server_stop",
 )
 
 
@@ -83,6 +85,9 @@ def lib():
             "lake_linnos_capture": (ctypes.c_int, [P, P, P, I64, P, P, SZ, P]),
             "lake_linnos_auto_threshold": (ctypes.c_int, [I32, P]),
             "lake_linnos_set_auto_threshold": (ctypes.c_int, [I32, I64]),
+            "lake_linnos_server_start": (ctypes.c_int, [I32, P]),
+            "lake_linnos_server_infer": (ctypes.c_int, [P, P, I32, P, P]),
+            "lake_linnos_server_stop": (ctypes.c_int, [P]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -230,3 +235,26 @@ def auto_threshold(arch: int) -> int:
 
 def set_auto_threshold(arch: int, n_min: int) -> None:
     _check(lib().lake_linnos_set_auto_threshold(arch, n_min), "set_auto_threshold")
+
+
+class Server:
+    """Persistent resident-weights server (lake_linnos_server_*): host buffers in and out."""
+
+    def __init__(self, model_id: int):
+        self._h = ctypes.c_void_p(0)
+        _check(lib().lake_linnos_server_start(model_id, ctypes.byref(self._h)), "server_start")
+
+    def infer(self, h_raw, n: int, h_decisions, h_logits=None) -> None:
+        _check(lib().lake_linnos_server_infer(self._h, _ptr(h_raw), n, _ptr(h_decisions),
+                                              _ptr(h_logits)), "server_infer")
+
+    def stop(self) -> None:
+        if self._h:
+            _check(lib().lake_linnos_server_stop(self._h), "server_stop")
+            self._h = ctypes.c_void_p(0)
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.stop()

@@ -397,3 +397,38 @@ def test_auto_policy_routes_by_arch_and_size():
         assert np.array_equal(lg3.view(np.uint32), r3.view(np.uint32))
     finally:
         lake.set_auto_threshold(2, lake.LAKE_AUTO_TC_MIN_N[2])
+
+
+# ------------------------------------------------------------------------- persistent server
+@pytest.mark.parametrize("arch", ARCHS)
+def test_server_bit_exact_batches(arch):
+    import torch
+    raw = _trace(2000, seed=123)
+    blob = inputs.weights(arch, 10 + arch)
+    rlg, rdec = oracle.infer_raw(arch, blob, raw, nthreads=0)
+    h_dec = np.zeros(lake.LAKE_SERVER_MAX_BATCH, np.uint8)
+    h_lg = np.zeros((lake.LAKE_SERVER_MAX_BATCH, 2), np.float32)
+    rng = np.random.default_rng(arch)
+    with lake.Server(10 + arch) as srv:
+        pos = 0
+        for b in [1, 2, 64, 17, 63, 8, 1, 33] + list(rng.integers(1, 65, size=30)):
+            b = int(b)
+            chunk = np.ascontiguousarray(raw[pos:pos + b])
+            srv.infer(chunk, b, h_dec, h_lg)
+            assert np.array_equal(h_dec[:b], rdec[pos:pos + b])
+            assert np.array_equal(h_lg[:b].view(np.uint32), rlg[pos:pos + b].view(np.uint32))
+            pos += b
+        with pytest.raises(lake.LakeError):
+            srv.infer(raw, lake.LAKE_SERVER_MAX_BATCH + 1, h_dec, h_lg)
+
+
+def test_server_survives_unload():
+    lake.load_weights(555, 2, inputs.weights(2, 555), 0)
+    srv = lake.Server(555)
+    lake.unload(555, 0)  # the server keeps its own copy of the weights
+    raw = _trace(10, seed=5)
+    h_dec = np.zeros(10, np.uint8)
+    srv.infer(np.ascontiguousarray(raw), 10, h_dec)
+    srv.stop()
+    _, rdec = oracle.infer_raw(2, inputs.weights(2, 555), raw, nthreads=0)
+    assert np.array_equal(h_dec, rdec)
