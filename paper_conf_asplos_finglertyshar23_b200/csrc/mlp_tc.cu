@@ -63,6 +63,12 @@ enum TraceKind { T_XFULL = 1, T_TEMPTY = 2, T_HREADY = 3, T_COMMIT = 4, T_DFULL 
                  T_CHUNK = 6, T_LAYER_END = 7, T_XEMPTY = 8, T_XARRIVE = 9, T_ISSUED = 10,
                  T_LDWAIT = 11, T_STS = 12, T_FENCE = 13 };
 
+// H (the next layer's A operand) stays in tensor memory, packed in place into the
+// accumulator it came from (default); -DLAKE_H_SMEM restores the SMEM H tile + proxy fences.
+#ifndef LAKE_H_SMEM
+#define LAKE_H_TMEM 1
+#endif
+
 namespace lake {
 namespace {
 
@@ -198,6 +204,35 @@ __device__ __forceinline__ void epi_to_h(const uint32_t (&r)[W], const uint32_t 
     }
     ptx::st_shared_v4(hrow_addr + ((col0 >> 3) + gq) * kLboR128, p[0], p[1], p[2], p[3]);
   }
+}
+
+// Same conversion, but the packed pairs go back into tensor memory, in place: the warp's
+// own W fp32 columns [col0, col0+W) (just read) become W/2 packed columns [col0, col0+W/2),
+// which the next layer's MMA reads as its A operand (H kept in TMEM, no SMEM / proxy fence).
+// K-step s (features 16s..16s+15) therefore sits at packed column tmem_a_col(s).
+template <int PREC, int W>
+__device__ __forceinline__ void epi_to_h_tmem(const uint32_t (&r)[W], const uint32_t *bias2,
+                                              uint32_t col0, uint32_t tlane_base) {
+  const uint32_t one2 = PREC == 0 ? 0x3C003C00u : 0x3F803F80u;
+  uint32_t p[W / 2];
+#pragma unroll
+  for (int gq = 0; gq < W / 8; ++gq) {
+    const uint4 bb = *reinterpret_cast<const uint4 *>(bias2 + (col0 >> 1) + gq * 4);
+    const uint32_t bv[4] = {bb.x, bb.y, bb.z, bb.w};
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      const int c = gq * 8 + e * 2;
+      const float v0 = __uint_as_float(r[c]), v1 = __uint_as_float(r[c + 1]);
+      p[gq * 4 + e] = PREC == 0 ? ptx::hfma2_relu_f16(ptx::pack_f16(v0, v1), one2, bv[e])
+                                : ptx::hfma2_relu_bf16(ptx::pack_bf16(v0, v1), one2, bv[e]);
+    }
+  }
+  if constexpr (W / 2 == 16) ptx::tmem_st_32x32b_x16(tlane_base + col0, p);
+  else ptx::tmem_st_32x32b_x8(tlane_base + col0, p);
+}
+
+__host__ __device__ constexpr uint32_t tmem_a_col(uint32_t s) {
+  return (s / (kEpiCols / 16)) * kEpiCols + (s % (kEpiCols / 16)) * 8;
 }
 
 // Last hidden layer: ReLU(acc + b) in fp32, accumulated straight into the two logits
@@ -367,7 +402,16 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
             h_phase ^= (1u << kc);
             LAKE_TEV(T_HREADY, it, l, kc);
             ptx::tc_fence_after();
-#ifdef LAKE_INLINE_DESC
+#ifdef LAKE_H_TMEM
+            // A = H(l-1), packed in place in the previous layer's accumulator buffer
+            const uint32_t ha = tmem + ((g - 1) & 1) * 256;
+            const uint64_t wd = l == 1 ? whdesc[1] : whdesc[2];
+#pragma unroll
+            for (uint32_t s = 0; s < kKStepsPerChunk; ++s) {
+              const uint32_t ks = kc * kKStepsPerChunk + s;
+              ptx::mma_f16_cg2_ts(d, ha + tmem_a_col(ks), wd + ks * kStep, idesc, ks);
+            }
+#elif defined(LAKE_INLINE_DESC)
 #pragma unroll
             for (uint32_t s = 0; s < kKStepsPerChunk; ++s) {
               const uint32_t ks = kc * kKStepsPerChunk + s;
@@ -526,6 +570,11 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         constexpr bool kPrefetch = W <= 32;  // two W-register buffers
 #endif
         uint32_t ra[W], rb[W];  // rb unused (eliminated) without prefetch
+#ifdef LAKE_H_TMEM
+#define EPI_H(R) epi_to_h_tmem<PREC, W>(R, prm2 + l * kHidden / 2, col0, tbase)
+#else
+#define EPI_H(R) epi_to_h<PREC, W>(R, prm2 + l * kHidden / 2, col0, hrow)
+#endif
         ptx::tmem_ld_cols<W>(tbase + col_of(0), ra);
         ptx::tmem_ld_wait();
         if (!last) {
@@ -539,17 +588,22 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
                 if (j & 1) ptx::tmem_ld_cols<W>(tbase + col_of(j + 1), ra);
                 else ptx::tmem_ld_cols<W>(tbase + col_of(j + 1), rb);
               }
-              if (j & 1) epi_to_h<PREC, W>(rb, prm2 + l * kHidden / 2, col0, hrow);
-              else epi_to_h<PREC, W>(ra, prm2 + l * kHidden / 2, col0, hrow);
+              if (j & 1) EPI_H(rb);
+              else EPI_H(ra);
             } else {
               if (j > 0) {
                 ptx::tmem_ld_cols<W>(tbase + col0, ra);
                 ptx::tmem_ld_wait();
               }
-              epi_to_h<PREC, W>(ra, prm2 + l * kHidden / 2, col0, hrow);
+              EPI_H(ra);
             }
             LAKE_TEV(T_STS, it, l, kc);
+#ifdef LAKE_H_TMEM
+            ptx::tmem_st_wait();
+            ptx::tc_fence_before();
+#else
             ptx::fence_proxy_async_smem();
+#endif
             LAKE_TEV(T_FENCE, it, l, kc);
             __syncwarp();
             if (lane == 0) ptx::mbar_arrive_cluster(hready_leader0 + kc * 8);
