@@ -105,7 +105,11 @@ constexpr uint32_t kHreadyCount = 2 * kGroupWarps;     // the H group's warps, b
 #endif
 constexpr uint32_t kKStepsPerChunk = kChunkCols / 16;
 constexpr int kThreads = 32 * (3 + kEpiWarps + 1);  // digitisers(2) + loader + epi + MMA
-constexpr uint32_t kHBytes = 128 * kHidden * 2;   // 64 KB
+#ifdef LAKE_H_TMEM
+constexpr uint32_t kHBytes = 0;                   // H lives in TMEM
+#else
+constexpr uint32_t kHBytes = 128 * kHidden * 2;   // 64 KB SMEM H tile
+#endif
 constexpr uint32_t kXBytes = 128 * kTcK0 * 2;     // 8 KB
 constexpr uint32_t kLboR128 = 128 * 16;           // K-direction core stride, 128-row operand
 constexpr uint32_t kPrmFloats = kHidden + 2 * kHidden + 4;  // last-layer bias | W_out | b_out
