@@ -52,12 +52,14 @@ def parse():
     p.add_argument("--config", default="C5", choices=["C1", "C3", "C4", "C5"])
     p.add_argument("--prec", default=None, choices=["fp32", "f16", "bf16"])
     p.add_argument("--arch", type=int, default=None)
-    p.add_argument("--n", type=int, default=None)
-    p.add_argument("--mode", default="throughput", choices=["throughput", "sweep"])
+    p.add_argument("--n-ios", dest="n", type=int, default=None)
+    p.add_argument("--mode", default="throughput", choices=["throughput", "sweep", "report"])
     p.add_argument("--sweep-out", default=None)
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=12.0)
+    p.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                   help="control-plane backend (gloo: lets a 1-GPU box run several ranks)")
     return p.parse_args()
 
 
@@ -90,6 +92,8 @@ def max_over_ranks(x: float, dist, device=None) -> float:
     if dist is None:
         return x
     import torch
+    if dist.get_backend() == "gloo":
+        device = None  # gloo reduces host tensors
     t = torch.tensor([x], dtype=torch.float64, device=device)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
@@ -222,7 +226,10 @@ def run_ours(args):
     world, rank, local = dist_env()
     if args.gpus != world and world > 1:
         log(f"warning: --gpus {args.gpus} but WORLD_SIZE {world}")
-    dist = dist_init(world, local)
+    # testing aid: BENCH_SAME_DEVICE=1 puts every rank on GPU 0 (with --dist-backend gloo)
+    if os.environ.get("BENCH_SAME_DEVICE") == "1":
+        local = 0
+    dist = dist_init(world, local, args.dist_backend)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     from paper_conf_asplos_finglertyshar23_b200 import lake
@@ -489,12 +496,110 @@ def run_sweep(args):
                       "crossovers": [r for r in out if "crossover_batch" in r]}))
 
 
+# ------------------------------------------------------------------ C3 / C4 report
+def run_report(args):
+    """BASELINE configs[2] (C3: NN+1 / NN+2, 2^20 I/Os, tensor cores vs FP32) and configs[3]
+    (C4: 3 per-SSD models interleaved, 2^22 I/Os, grouping overhead): throughput, fraction of
+    the relevant peak, and accuracy of the tensor paths against the oracle on a sample."""
+    import torch
+    import oracle
+    from paper_conf_asplos_finglertyshar23_b200 import lake
+    torch.cuda.set_device(0)
+    dev = torch.device("cuda", 0)
+    stream = torch.cuda.current_stream()
+    peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
+        os.path.join(ROOT, "MEASURED_PEAKS.json")) else {}
+    tpeak = peaks.get("bf16_tflops", 1590.0)
+    fpeak = 148 * 128 * 2 * peaks.get("sm_max_mhz", 1965.0) * 1e6 / 1e12
+    rows = []
+
+    def timed(fn, reps=10):
+        for _ in range(3):
+            fn()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(reps):
+            fn()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) / reps
+
+    # ---- C3
+    n = 1 << 20
+    raw = inputs.workload("C3", n=n)["raw"]
+    x = torch.from_numpy(raw.view(np.int32)).to(dev)
+    dec = torch.empty(n, dtype=torch.uint8, device=dev)
+    lg = torch.empty((n, 2), dtype=torch.float32, device=dev)
+    smp = np.random.default_rng(0).choice(n, 8192, replace=False)
+    for arch in (1, 2):
+        blob = inputs.weights(arch, 0)
+        lake.load_weights(60 + arch, arch, blob, 0)
+        rlg, rdec = oracle.infer_raw(arch, blob, raw[smp], nthreads=0)
+        ref = rlg.astype(np.float64)
+        rms = np.sqrt(np.mean(ref ** 2))
+        for prec in ("fp32", "f16", "bf16"):
+            flags = lake.LAKE_IN_RAW | lake.PREC_FLAGS[prec]
+            ms = timed(lambda: lake.infer(x, flags, n, 60 + arch, dec, lg, stream))
+            lake.infer(x, flags, n, 60 + arch, dec, lg, stream)
+            torch.cuda.synchronize()
+            d = dec.cpu().numpy()[smp]
+            l = lg.cpu().numpy()[smp].astype(np.float64)
+            rel = np.abs(l - ref) / np.maximum(np.abs(ref), rms)
+            dis = d != rdec
+            tflops = ARCH_FLOPS[arch] * n / (ms / 1e3) / 1e12
+            rows.append(dict(config="C3", arch=ARCH_NAME[arch], path=prec, n=n,
+                             ms=round(ms, 4), inferences_per_s=round(n / (ms / 1e3), 1),
+                             tflops=round(tflops, 2),
+                             frac_of_peak=round(tflops / (fpeak if prec == "fp32" else tpeak), 4),
+                             peak=("FP32 %.1f TF/s (derived)" % fpeak) if prec == "fp32"
+                             else "bf16 %.1f TF/s (measured)" % tpeak,
+                             sample=int(smp.size), agreement=float(1 - dis.mean()),
+                             max_rel_err=float(rel.max()),
+                             max_disagree_margin=float(np.abs(ref[dis, 0] - ref[dis, 1]).max()) if dis.any() else 0.0,
+                             margin_sd=float(np.std(ref[:, 1] - ref[:, 0]))))
+            log(json.dumps(rows[-1]))
+        lake.unload(60 + arch, 0)
+    # ---- C4
+    n = 1 << 22
+    w = inputs.workload("C4", n=n)
+    x = torch.from_numpy(w["raw"].view(np.int32)).to(dev)
+    ids = torch.from_numpy(w["model_ids"]).to(dev)
+    dec = torch.empty(n, dtype=torch.uint8, device=dev)
+    wsb = lake.workspace_bytes(n)
+    ws = torch.empty(wsb, dtype=torch.uint8, device=dev)
+    for m, (a, blob) in w["models"].items():
+        lake.load_weights(m, a, blob, 0)
+    flags = lake.LAKE_IN_RAW | lake.LAKE_PREC_F16
+    t_multi = timed(lambda: lake.infer_multi(x, flags, n, ids, dec, None, ws, wsb, stream))
+    t_group = timed(lambda: lake.multi_group(n, ids, ws, wsb, stream))
+    mids = w["model_ids"]
+    parts = [torch.from_numpy(np.ascontiguousarray(w["raw"][mids == m]).view(np.int32)).to(dev)
+             for m in range(3)]
+    t_split = timed(lambda: [lake.infer(p, flags, p.shape[0], m, dec, None, stream)
+                             for m, p in enumerate(parts)])
+    rows.append(dict(config="C4", arch=ARCH_NAME[2], path="f16", n=n, models=3,
+                     infer_multi_ms=round(t_multi, 4), group_ms=round(t_group, 4),
+                     presplit_3_infer_ms=round(t_split, 4),
+                     inferences_per_s=round(n / (t_multi / 1e3), 1),
+                     grouping_overhead=round(t_multi / t_split - 1, 4)))
+    log(json.dumps(rows[-1]))
+    path = args.sweep_out or os.path.join(ROOT, "gpurun_out", "report.jsonl")
+    os.makedirs(os.path.dirname(path), exist_ok=True)
+    with open(path, "w") as f:
+        for r in rows:
+            f.write(json.dumps(r) + "\n")
+    print(json.dumps({"metric": "C3/C4 report", "rows": len(rows)}))
+
+
 def main():
     args = parse()
     if args.impl == "reference":
         run_reference(args)
     elif args.mode == "sweep":
         run_sweep(args)
+    elif args.mode == "report":
+        run_report(args)
     else:
         run_ours(args)
 

@@ -1,0 +1,51 @@
+"""Small invocation of every kernel, for compute-sanitizer:
+digitise, FP32 (16- and 64-row tiles), tcgen05 fp16/bf16, multi-model grouping, capture,
+host pipeline (zero-copy + chunked), persistent server."""
+import os
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+from paper_conf_asplos_finglertyshar23_b200 import inputs, lake  # noqa: E402
+
+torch.cuda.set_device(0)
+dev = "cuda:0"
+raw = inputs.edge_raw(3000, seed=1)
+x = torch.from_numpy(raw.view(np.int32)).to(dev)
+for m, a in ((1, 0), (2, 1), (3, 2)):
+    lake.load_weights(m, a, inputs.weights(a, m), 0)
+d = torch.empty((3000, 32), dtype=torch.uint8, device=dev)
+lake.digitize(x, 129, d)
+dec = torch.empty(3000, dtype=torch.uint8, device=dev)
+lg = torch.empty((3000, 2), dtype=torch.float32, device=dev)
+for n in (1, 129, 3000):
+    for f in (lake.LAKE_PREC_FP32, lake.LAKE_PREC_F16, lake.LAKE_PREC_BF16):
+        lake.infer(x, lake.LAKE_IN_RAW | f, n, 3, dec, lg)
+lake.infer(d, lake.LAKE_IN_DIGITS | lake.LAKE_PREC_F16, 129, 2, dec, lg)
+ids = torch.from_numpy(np.random.default_rng(0).integers(1, 4, 3000).astype(np.int32)).to(dev)
+wsb = lake.workspace_bytes(3000)
+ws = torch.empty(wsb, dtype=torch.uint8, device=dev)
+lake.infer_multi(x, lake.LAKE_IN_RAW | lake.LAKE_PREC_F16, 3000, ids, dec, lg, ws, wsb)
+lake.infer_multi(x, lake.LAKE_IN_RAW | lake.LAKE_PREC_FP32, 3000, ids, dec, lg, ws, wsb)
+tr = inputs.device_trace("azure", 1000, 3, 3.0)
+a = torch.from_numpy(tr["arrival_ns"]).to(dev)
+c = torch.from_numpy(tr["complete_ns"]).to(dev)
+out = torch.empty((1000, 9), dtype=torch.int32, device=dev)
+cwb = lake.capture_workspace_bytes(1000)
+cws = torch.empty(cwb, dtype=torch.uint8, device=dev)
+lake.capture(a, c, None, 1000, out, cws, cwb)
+h_in = torch.from_numpy(raw.view(np.int32)).pin_memory()
+h_dec = torch.empty(3000, dtype=torch.uint8).pin_memory()
+sb = lake.host_staging_bytes(3000, lake.LAKE_IN_RAW)
+stg = torch.empty(sb, dtype=torch.uint8, device=dev)
+lake.infer_host(h_in, lake.LAKE_IN_RAW | lake.LAKE_PREC_F16, 3000, 3, None, h_dec, None, stg, sb)
+torch.cuda.synchronize()
+if os.environ.get("SANITIZE_SERVER", "1") == "1":
+    with lake.Server(3) as srv:
+        hd = np.zeros(64, np.uint8)
+        srv.infer(np.ascontiguousarray(raw[:5]), 5, hd)
+        srv.infer(np.ascontiguousarray(raw[:64]), 64, hd)
+torch.cuda.synchronize()
+print("sanitize run ok")
