@@ -49,8 +49,8 @@ __device__ unsigned long long *g_lake_trace = nullptr;
 #define LAKE_TRACE_CAP (1u << 16)
 #define LAKE_TEV(kind, tile, layer, chunk)                                                   \
   do {                                                                                    \
-    if (g_lake_trace && cid == 0 && rank == 0 && tr_stream >= 0 && tr_i < LAKE_TRACE_CAP) { \
-      unsigned long long *p_ = g_lake_trace + 2ull * (tr_stream * LAKE_TRACE_CAP + tr_i++);  \
+    if (tr_stream >= 0 && tr_i < LAKE_TRACE_CAP) {                                        \
+      unsigned long long *p_ = tr_buf + 2ull * (tr_stream * LAKE_TRACE_CAP + tr_i++);        \
       p_[0] = ((unsigned long long)(kind) << 56) | ((unsigned long long)(tile) << 24) |     \
               ((unsigned long long)(layer) << 8) | (unsigned long long)(chunk);              \
       p_[1] = clock64();                                                                  \
@@ -227,12 +227,21 @@ __device__ __forceinline__ void epi_to_h_tmem(const uint32_t (&r)[W], const uint
     for (int e = 0; e < 4; ++e) {
       const int c = gq * 8 + e * 2;
       const float v0 = __uint_as_float(r[c]), v1 = __uint_as_float(r[c + 1]);
+#ifdef LAKE_ABL_NOCVT  // timing-only ablation: no conversion arithmetic
+      p[gq * 4 + e] = r[c] ^ r[c + 1] ^ bv[e];
+#else
       p[gq * 4 + e] = PREC == 0 ? ptx::hfma2_relu_f16(ptx::pack_f16(v0, v1), one2, bv[e])
                                 : ptx::hfma2_relu_bf16(ptx::pack_bf16(v0, v1), one2, bv[e]);
+#endif
     }
   }
-  if constexpr (W / 2 == 16) ptx::tmem_st_32x32b_x16(tlane_base + col0, p);
-  else ptx::tmem_st_32x32b_x8(tlane_base + col0, p);
+#ifdef LAKE_ABL_NOST  // timing-only ablation: H not written back (never true at run time)
+  if (p[0] == 0x12345678u && p[1] == 0x9abcdef0u)
+#endif
+  {
+    if constexpr (W / 2 == 16) ptx::tmem_st_32x32b_x16(tlane_base + col0, p);
+    else ptx::tmem_st_32x32b_x8(tlane_base + col0, p);
+  }
 }
 
 __host__ __device__ constexpr uint32_t tmem_a_col(uint32_t s) {
@@ -254,10 +263,14 @@ __device__ __forceinline__ void epi_to_logits(const uint32_t (&r)[W], const floa
     const float ww1[4] = {w1.x, w1.y, w1.z, w1.w};
 #pragma unroll
     for (int e = 0; e < 4; ++e) {
+#ifdef LAKE_ABL_NOLOGITS  // timing-only ablation: no output-layer arithmetic
+      p[e] += __uint_as_float(r[c4 * 4 + e]) + bb[e] + ww0[e] + ww1[e];
+#else
       float h = __uint_as_float(r[c4 * 4 + e]) + bb[e];
       h = h > 0.0f ? h : 0.0f;
       p[(e & 1) * 2 + 0] = fmaf(h, ww0[e], p[(e & 1) * 2 + 0]);
       p[(e & 1) * 2 + 1] = fmaf(h, ww1[e], p[(e & 1) * 2 + 1]);
+#endif
     }
   }
 }
@@ -276,7 +289,9 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
   const uint32_t cid = ptx::cluster_id_x(), ncl = ptx::num_clusters_x();
 
 #ifdef LAKE_TRACE
-  const int tr_stream = (warp == kWarpMma && lane == 0) ? 0 : (warp == kWarpEpi && lane == 0) ? 1
+  unsigned long long *const tr_buf = g_lake_trace;  // read once: events cost no global load
+  const int tr_stream = !(tr_buf && cid == 0 && rank == 0) ? -1
+                      : (warp == kWarpMma && lane == 0) ? 0 : (warp == kWarpEpi && lane == 0) ? 1
                       : (warp == kWarpMma - 1 && lane == 0) ? 2 : (threadIdx.x == 0) ? 3 : -1;
   uint32_t tr_i = 0;
 #endif
@@ -339,7 +354,11 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
   } else if (warp == kWarpMma) {
     // ================= MMA issuer (leader CTA, one thread) =================
     if (rank == 0 && lane == 0) {
+#ifdef LAKE_ABL_HALFN  // timing-only ablation: hidden-layer MMAs with N = 128 (half the work)
+      const uint32_t idesc = ptx::umma_idesc_f16(PREC, 256, 128);
+#else
       const uint32_t idesc = ptx::umma_idesc_f16(PREC, 256, 256);
+#endif
       // descriptors: advancing K by 16 elements = +2 core matrices = +2*LBO bytes, i.e.
       // +(2*LBO)>>4 in the 14-bit start-address field (no carry: SMEM < 256 KB)
       constexpr uint64_t kStep = (2 * kLboR128) >> 4;

@@ -1,11 +1,13 @@
 // Microbenchmark: tcgen05.ld (32x32b.x32) latency and TMEM->RF bandwidth with and without
-// concurrent tcgen05.mma traffic (cta_group::2, M=256, N=128, A from TMEM, B from SMEM).
+// concurrent tcgen05.mma traffic (cta_group::2, M=256, N=128, A from TMEM, B from SMEM), and
+// the MMA rate itself while the load warps run (ST=1: each load is followed by a 16-column
+// tcgen05.st, the H write-back of the fused kernel).
 #include <cstdio>
 #include <cstdint>
 #include "../../paper_conf_asplos_finglertyshar23_b200/csrc/lake_ptx.cuh"
 using namespace lake;
 
-template <int WITH_MMA, int NLD_WARPS>
+template <int WITH_MMA, int NLD_WARPS, int ST = 0>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(32 * (NLD_WARPS + 1), 1)
 k(unsigned long long *out, int iters) {
   extern __shared__ __align__(1024) uint8_t smem[];
@@ -26,11 +28,15 @@ k(unsigned long long *out, int iters) {
     if (WITH_MMA && rank == 0 && lane == 0) {
       const uint32_t idesc = ptx::umma_idesc_f16(0, 256, 128) | (1u << 16);
       const uint64_t bdesc = ptx::umma_desc(sb, 1024, 128);
-      for (int i = 0; i < 64 * iters; ++i) {
+      const unsigned long long m0 = clock64();
+      for (int i = 0; i < 16 * iters; ++i) {
         const uint32_t ks = i & 15;
         ptx::mma_f16_cg2_ts(tmem + 256 + ((i >> 4) & 1) * 128, tmem + ks * 8, bdesc + ks * 128, idesc, ks);
       }
       ptx::mma_commit_cg2(bar, 0x3);
+      ptx::mbar_wait(bar, 0);
+      out[126] = (clock64() - m0);
+      out[127] = 16ull * iters;
     }
   } else {
     // loads from columns the MMA does not write (the A region 0..255)
@@ -44,6 +50,13 @@ k(unsigned long long *out, int iters) {
       const unsigned long long a = clock64();
       ptx::tmem_ld_32x32b_x32(ta + (i & 3) * 64, r);
       ptx::tmem_ld_wait();
+      if (ST) {
+        uint32_t w[16];
+#pragma unroll
+        for (int j = 0; j < 16; ++j) w[j] = r[j] ^ r[j + 16];
+        ptx::tmem_st_32x32b_x16(ta + (i & 3) * 64 + 128, w);
+        ptx::tmem_st_wait();
+      }
 #pragma unroll
       for (int j = 0; j < 32; ++j) acc += r[j];
       lat += clock64() - a;
@@ -55,19 +68,19 @@ k(unsigned long long *out, int iters) {
     }
     if (acc == 0xdeadbeef) out[100] = acc;
   }
-  if (WITH_MMA && threadIdx.x == 0) ptx::mbar_wait(bar, 0);
+  if (WITH_MMA && threadIdx.x == 0 && rank == 1) ptx::mbar_wait(bar, 0);
   __syncwarp();
   ptx::tc_fence_before();
   ptx::cluster_sync();
   if (warp == 0) { ptx::tc_fence_after(); ptx::tmem_dealloc_cg2(tmem, 512); }
 }
 
-template <int WITH_MMA, int NW>
+template <int WITH_MMA, int NW, int ST = 0>
 void run(const char *name) {
   unsigned long long *d, h[64] = {};
   cudaMalloc(&d, 8 * 128);
   cudaMemset(d, 0, 8 * 128);
-  auto f = k<WITH_MMA, NW>;
+  auto f = k<WITH_MMA, NW, ST>;
   cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 70 * 1024);
   const int iters = 2000;
   for (int rep = 0; rep < 2; ++rep) {
@@ -75,11 +88,15 @@ void run(const char *name) {
     cudaError_t e = cudaDeviceSynchronize();
     if (e != cudaSuccess) { printf("%s: %s\n", name, cudaGetErrorString(e)); return; }
   }
+  unsigned long long hm[2] = {};
   cudaMemcpy(h, d, 8 * 64, cudaMemcpyDeviceToHost);
+  cudaMemcpy(hm, d + 126, 16, cudaMemcpyDeviceToHost);
   double bw = 0;
   unsigned long long lat = 0;
   for (int w = 0; w < NW; ++w) { lat += h[w * 2]; bw += 4096.0 * iters / h[w * 2 + 1]; }
-  printf("%-24s %2d ld warps: ld x32 latency %5llu cycles, TMEM->RF %6.0f B/clk/SM\n", name, NW, lat / NW, bw);
+  printf("%-24s %2d ld warps: ld x32 latency %5llu cycles, TMEM->RF %6.0f B/clk/SM", name, NW, NW ? lat / (NW ? NW : 1) : 0ull, bw);
+  if (WITH_MMA) printf(", MMA %.1f cycles each (64 = full rate)", (double)hm[0] / hm[1]);
+  printf("\n");
   cudaFree(d);
 }
 
@@ -90,5 +107,8 @@ int main() {
   run<1, 8>("with MMA");
   run<0, 16>("no MMA");
   run<1, 16>("with MMA");
+  run<1, 0>("MMA alone");
+  run<1, 8, 1>("with MMA, ld+st");
+  run<1, 16, 1>("with MMA, ld+st");
   return 0;
 }
