@@ -427,6 +427,7 @@ def run_sweep(args):
         for prec in ("fp32", "f16", "bf16"):
             flags = lake.LAKE_IN_RAW | lake.PREC_FLAGS[prec]
             cross = None
+            gcross = None
             scross = None
             for b in sizes:
                 raw = np.ascontiguousarray(raw_all[:b])
@@ -447,6 +448,31 @@ def run_sweep(args):
                     t0 = time.perf_counter()
                     once()
                     ts.append((time.perf_counter() - t0) * 1e6)
+                # CUDA-Graph variant (C2): H2D copy, fused kernel and D2H copy captured once,
+                # each batch one graph replay + stream sync (launch overheads amortised)
+                gs = torch.cuda.Stream()
+                g_dec = torch.empty(b, dtype=torch.uint8).pin_memory()
+                with torch.cuda.stream(gs):
+                    lake.infer(d_in, flags, b, 40 + arch, d_dec, None, gs)  # warm (attributes)
+                gs.synchronize()
+                graph = torch.cuda.CUDAGraph()
+                with torch.cuda.graph(graph, stream=gs):
+                    d_in.copy_(h_in, non_blocking=True)
+                    lake.infer(d_in, flags, b, 40 + arch, d_dec, None, gs)
+                    g_dec.copy_(d_dec, non_blocking=True)
+                gt = []
+                with torch.cuda.stream(gs):  # replay() launches on the current stream
+                    for _ in range(warm):
+                        graph.replay()
+                        gs.synchronize()
+                    for _ in range(reps):
+                        t0 = time.perf_counter()
+                        graph.replay()
+                        gs.synchronize()
+                        gt.append((time.perf_counter() - t0) * 1e6)
+                if not np.array_equal(g_dec.numpy(), h_dec.numpy()):
+                    raise RuntimeError(f"graph replay differs from infer_host (arch {arch} {prec} b={b})")
+                del graph
                 ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 ev0.record(stream)
                 for _ in range(reps):
@@ -461,10 +487,15 @@ def run_sweep(args):
                     oracle.infer_raw(arch, blob, raw, nthreads=1)
                 cpu_us = (time.perf_counter() - t0) * 1e6 / oreps
                 med = float(np.median(ts))
+                gmed = float(np.median(gt))
                 if cross is None and med < cpu_us:
                     cross = b
+                if gcross is None and gmed < cpu_us:
+                    gcross = b
                 row = dict(arch=ARCH_NAME[arch], prec=prec, batch=b, e2e_us_median=round(med, 2),
                            e2e_us_p99=round(float(np.percentile(ts, 99)), 2),
+                           graph_us_median=round(gmed, 2),
+                           graph_us_p99=round(float(np.percentile(gt, 99)), 2),
                            device_us=round(dev_us, 2), cpu_1thread_us=round(cpu_us, 2))
                 if prec == "fp32" and b <= lake.LAKE_SERVER_MAX_BATCH:
                     # NEXT-2: persistent resident-weights server (doorbell, no launch/copies)
@@ -484,6 +515,7 @@ def run_sweep(args):
                 out.append(row)
                 log(json.dumps(row))
             out.append(dict(arch=ARCH_NAME[arch], prec=prec, crossover_batch=cross,
+                            graph_crossover_batch=gcross,
                             **({"server_crossover_batch": scross} if prec == "fp32" else {})))
             log(json.dumps(out[-1]))
         lake.unload(40 + arch, 0)

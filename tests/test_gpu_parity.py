@@ -142,6 +142,42 @@ def test_batch_independence(prec):
     assert np.array_equal(full[1], np.concatenate([a[1], b[1]]))
 
 
+@pytest.mark.parametrize("prec", [lake.LAKE_PREC_F16, lake.LAKE_PREC_FP32])
+def test_cuda_graph_capture(prec):
+    # the C ABI calls are capturable into a CUDA graph (C2's graph variant): H2D, fused
+    # kernel, D2H replayed on new inputs give exactly the direct call's results
+    import torch
+    n = 777
+    raw_a, raw_b = _trace(n, seed=61), _trace(n, seed=62)
+    flags = lake.LAKE_IN_RAW | prec
+    h_in = torch.from_numpy(raw_a.view(np.int32).copy()).pin_memory()
+    d_in = torch.empty_like(h_in, device="cuda:0")
+    d_dec = torch.empty(n, dtype=torch.uint8, device="cuda:0")
+    d_lg = torch.empty((n, 2), dtype=torch.float32, device="cuda:0")
+    h_dec = torch.empty(n, dtype=torch.uint8).pin_memory()
+    h_lg = torch.empty((n, 2), dtype=torch.float32).pin_memory()
+    s = torch.cuda.Stream()
+    d_in.copy_(h_in)
+    lake.infer(d_in, flags, n, 12, d_dec, d_lg, s)  # warm-up outside the capture
+    s.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        d_in.copy_(h_in, non_blocking=True)
+        lake.infer(d_in, flags, n, 12, d_dec, d_lg, s)
+        h_dec.copy_(d_dec, non_blocking=True)
+        h_lg.copy_(d_lg, non_blocking=True)
+    for raw in (raw_a, raw_b):
+        h_in.copy_(torch.from_numpy(raw.view(np.int32)))
+        h_dec.fill_(9)
+        with torch.cuda.stream(s):  # replay() launches on the current stream
+            g.replay()
+        s.synchronize()  # only the graph's own stream: its D2H must have landed
+        got_dec, got_lg = h_dec.numpy().copy(), h_lg.numpy().copy()
+        lg, dec = run_infer(12, raw, flags)
+        assert np.array_equal(got_dec, dec)
+        assert np.array_equal(got_lg.view(np.uint32), lg.view(np.uint32))
+
+
 # ------------------------------------------------------------------------- multi-model
 @pytest.fixture(scope="module")
 def multi_models():
