@@ -530,9 +530,10 @@ def run_sweep(args):
 
 # ------------------------------------------------------------------ C3 / C4 report
 def run_report(args):
-    """BASELINE configs[2] (C3: NN+1 / NN+2, 2^20 I/Os, tensor cores vs FP32) and configs[3]
-    (C4: 3 per-SSD models interleaved, 2^22 I/Os, grouping overhead): throughput, fraction of
-    the relevant peak, and accuracy of the tensor paths against the oracle on a sample."""
+    """BASELINE configs[2] (C3: NN+1 / NN+2, 2^20 I/Os, tensor cores vs FP32), configs[3]
+    (C4: 3 per-SSD models interleaved, 2^22 I/Os, every arch, grouping overhead) and
+    configs[4] on one GPU (C5: 64 NN+2 models, 2^24 I/Os, fp16 / bf16 / FP32): throughput,
+    fraction of the relevant peak, and accuracy against the oracle on a sample."""
     import torch
     import oracle
     from paper_conf_asplos_finglertyshar23_b200 import lake
@@ -592,36 +593,85 @@ def run_report(args):
                              margin_sd=float(np.std(ref[:, 1] - ref[:, 0]))))
             log(json.dumps(rows[-1]))
         lake.unload(60 + arch, 0)
-    # ---- C4
+    # ---- C4: 3 per-SSD models interleaved, every arch (headline NN+2 fp16)
     n = 1 << 22
-    w = inputs.workload("C4", n=n)
+    for arch in (2, 1, 0):
+        w = inputs.workload("C4", n=n, arch=arch)
+        x = torch.from_numpy(w["raw"].view(np.int32)).to(dev)
+        ids = torch.from_numpy(w["model_ids"]).to(dev)
+        dec = torch.empty(n, dtype=torch.uint8, device=dev)
+        wsb = lake.workspace_bytes(n)
+        ws = torch.empty(wsb, dtype=torch.uint8, device=dev)
+        for m, (a, blob) in w["models"].items():
+            lake.load_weights(m, a, blob, 0)
+        flags = lake.LAKE_IN_RAW | lake.LAKE_PREC_F16
+        t_multi = timed(lambda: lake.infer_multi(x, flags, n, ids, dec, None, ws, wsb, stream))
+        t_group = timed(lambda: lake.multi_group(n, ids, ws, wsb, stream))
+        mids = w["model_ids"]
+        parts = [torch.from_numpy(np.ascontiguousarray(w["raw"][mids == m]).view(np.int32)).to(dev)
+                 for m in range(3)]
+        t_split = timed(lambda: [lake.infer(p, flags, p.shape[0], m, dec, None, stream)
+                                 for m, p in enumerate(parts)])
+        rows.append(dict(config="C4", arch=ARCH_NAME[arch], path="f16", n=n, models=3,
+                         infer_multi_ms=round(t_multi, 4), group_ms=round(t_group, 4),
+                         presplit_3_infer_ms=round(t_split, 4),
+                         inferences_per_s=round(n / (t_multi / 1e3), 1),
+                         grouping_overhead=round(t_multi / t_split - 1, 4)))
+        log(json.dumps(rows[-1]))
+        for m in w["models"]:
+            lake.unload(m, 0)
+        del x, ids, dec, ws, parts
+    # ---- C5 on one GPU: 64 NN+2 models interleaved, 2^24 I/Os, every path (the throughput
+    # mode times the fp16 headline; here fp16, bf16 and FP32 with oracle-sample accuracy)
+    n = 1 << 24
+    w = inputs.workload("C5", n=n)
     x = torch.from_numpy(w["raw"].view(np.int32)).to(dev)
     ids = torch.from_numpy(w["model_ids"]).to(dev)
     dec = torch.empty(n, dtype=torch.uint8, device=dev)
+    lg = torch.empty((n, 2), dtype=torch.float32, device=dev)
     wsb = lake.workspace_bytes(n)
     ws = torch.empty(wsb, dtype=torch.uint8, device=dev)
     for m, (a, blob) in w["models"].items():
         lake.load_weights(m, a, blob, 0)
-    flags = lake.LAKE_IN_RAW | lake.LAKE_PREC_F16
-    t_multi = timed(lambda: lake.infer_multi(x, flags, n, ids, dec, None, ws, wsb, stream))
-    t_group = timed(lambda: lake.multi_group(n, ids, ws, wsb, stream))
-    mids = w["model_ids"]
-    parts = [torch.from_numpy(np.ascontiguousarray(w["raw"][mids == m]).view(np.int32)).to(dev)
-             for m in range(3)]
-    t_split = timed(lambda: [lake.infer(p, flags, p.shape[0], m, dec, None, stream)
-                             for m, p in enumerate(parts)])
-    rows.append(dict(config="C4", arch=ARCH_NAME[2], path="f16", n=n, models=3,
-                     infer_multi_ms=round(t_multi, 4), group_ms=round(t_group, 4),
-                     presplit_3_infer_ms=round(t_split, 4),
-                     inferences_per_s=round(n / (t_multi / 1e3), 1),
-                     grouping_overhead=round(t_multi / t_split - 1, 4)))
-    log(json.dumps(rows[-1]))
+    smp = np.random.default_rng(5).choice(n, 8192, replace=False)
+    mids = w["model_ids"][smp]
+    rlg = np.zeros((smp.size, 2), np.float32)
+    rdec = np.zeros(smp.size, np.uint8)
+    for m in np.unique(mids):
+        sel = mids == m
+        rlg[sel], rdec[sel] = oracle.infer_raw(2, w["models"][int(m)][1], w["raw"][smp[sel]], nthreads=0)
+    ref = rlg.astype(np.float64)
+    rms = np.sqrt(np.mean(ref ** 2))
+    for prec in ("f16", "bf16", "fp32"):
+        flags = lake.LAKE_IN_RAW | lake.PREC_FLAGS[prec]
+        ms = timed(lambda: lake.infer_multi(x, flags, n, ids, dec, lg, ws, wsb, stream),
+                   reps=10 if prec != "fp32" else 3)
+        lake.infer_multi(x, flags, n, ids, dec, lg, ws, wsb, stream)
+        torch.cuda.synchronize()
+        d = dec.cpu().numpy()[smp]
+        l = lg.cpu().numpy()[smp].astype(np.float64)
+        rel = np.abs(l - ref) / np.maximum(np.abs(ref), rms)
+        dis = d != rdec
+        tflops = ARCH_FLOPS[2] * n / (ms / 1e3) / 1e12
+        rows.append(dict(config="C5", arch=ARCH_NAME[2], path=prec, n=n, models=64,
+                         ms=round(ms, 4), inferences_per_s=round(n / (ms / 1e3), 1),
+                         tflops=round(tflops, 2),
+                         frac_of_peak=round(tflops / (fpeak if prec == "fp32" else tpeak), 4),
+                         peak=("FP32 %.1f TF/s (derived)" % fpeak) if prec == "fp32"
+                         else "bf16 %.1f TF/s (measured)" % tpeak,
+                         api="infer_multi (group + fused MLP), logits written",
+                         sample=int(smp.size), agreement=float(1 - dis.mean()),
+                         bit_exact_logits=bool(np.array_equal(l.astype(np.float32).view(np.uint32),
+                                                              rlg.view(np.uint32))),
+                         max_rel_err=float(rel.max()),
+                         max_disagree_margin=float(np.abs(ref[dis, 0] - ref[dis, 1]).max()) if dis.any() else 0.0))
+        log(json.dumps(rows[-1]))
     path = args.sweep_out or os.path.join(ROOT, "gpurun_out", "report.jsonl")
     os.makedirs(os.path.dirname(path), exist_ok=True)
     with open(path, "w") as f:
         for r in rows:
             f.write(json.dumps(r) + "\n")
-    print(json.dumps({"metric": "C3/C4 report", "rows": len(rows)}))
+    print(json.dumps({"metric": "C3/C4/C5 report", "rows": len(rows)}))
 
 
 def main():
