@@ -309,7 +309,11 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       ptx::mbar_init(bar(B_DFULLX + i), 1);      // tcgen05.commit (multicast): last layer
       ptx::mbar_init(bar(B_TEMPTY + i), 2 * kGroupWarps);  // the draining group, both CTAs
     }
+#ifdef LAKE_ABL_LOCALREADY  // timing-only ablation: chunk-ready counts only the leader's warps
+    for (uint32_t i = 0; i < kChunks; ++i) ptx::mbar_init(bar(B_HREADY + i), kHreadyCount / 2);
+#else
     for (uint32_t i = 0; i < kChunks; ++i) ptx::mbar_init(bar(B_HREADY + i), kHreadyCount);
+#endif
     ptx::mbar_init(bar(B_WFREE), 1);             // tcgen05.commit (multicast)
     ptx::fence_mbar_init();
   }
@@ -629,7 +633,11 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
 #endif
             LAKE_TEV(T_FENCE, it, l, kc);
             __syncwarp();
+#ifdef LAKE_ABL_LOCALREADY
+            if (lane == 0 && rank == 0) ptx::mbar_arrive_cluster(hready_leader0 + kc * 8);
+#else
             if (lane == 0) ptx::mbar_arrive_cluster(hready_leader0 + kc * 8);
+#endif
             LAKE_TEV(T_CHUNK, it, l, kc);
             if (kPrefetch && j + 1 < kWarpChunks) ptx::tmem_ld_wait();
             LAKE_TEV(T_LDWAIT, it, l, kc);
