@@ -13,6 +13,9 @@ citations and readings). Parity status per function:
                              invariants, numpy float64 GEMM chain)
 * ``capture``               pinned (hand-worked trace, heap-based event simulation of the
                              generator, invariants)
+* ``mlp_family``            pinned (NEXT-4: tiny integer ReLU MLPs vs int64 with C = 4
+                             and first-max ties, sigmoid special values and a float64
+                             chain, NaN / tie class rules, C = 2 against ``mlp``)
 * parity against the paper's trained model: unpinned (no weights/traces published).
 """
 from __future__ import annotations
@@ -62,6 +65,9 @@ def _load():
         lib.oracle_capture.restype = None
         lib.oracle_capture_rows.argtypes = [P, P, P, ctypes.c_int64, P, ctypes.c_int64, P]
         lib.oracle_capture_rows.restype = None
+        lib.oracle_mlp_family.argtypes = [ctypes.c_int, P, ctypes.c_int, P, P, ctypes.c_int64,
+                                          P, P, ctypes.c_int]
+        lib.oracle_mlp_family.restype = ctypes.c_int
         lib.oracle_max_threads.argtypes = []
         lib.oracle_max_threads.restype = ctypes.c_int
         _lib = lib
@@ -146,6 +152,24 @@ def infer_multi_raw(models: dict, raw: np.ndarray, model_ids: np.ndarray, nthrea
         logits[idx] = lg
         dec[idx] = d
     return logits, dec
+
+
+ACT_RELU, ACT_SIGMOID = 0, 1
+
+
+def mlp_family(widths, act: int, blob: np.ndarray, x: np.ndarray, nthreads: int = 1):
+    """NEXT-4 MLP family (MLLB / KML shapes): (out float32[n, C], classes int32[n])."""
+    widths = np.ascontiguousarray(widths, dtype=np.int32)
+    blob = np.ascontiguousarray(blob, dtype=np.float32)
+    x = np.ascontiguousarray(x, dtype=np.float32).reshape(-1, int(widths[0]))
+    n, C = x.shape[0], int(widths[-1])
+    out = np.zeros((n, C), dtype=np.float32)
+    cls = np.full(n, -1, dtype=np.int32)
+    rc = _load().oracle_mlp_family(len(widths) - 1, _ptr(widths), act, _ptr(blob), _ptr(x), n,
+                                   _ptr(out), _ptr(cls), nthreads)
+    if rc != 0:
+        raise ValueError(f"oracle_mlp_family failed ({rc})")
+    return out, cls
 
 
 def capture(arrival_ns: np.ndarray, complete_ns: np.ndarray, device=None) -> np.ndarray:

@@ -280,6 +280,69 @@ void oracle_capture_rows(const int64_t *a, const int64_t *c, const int32_t *dev,
     }
 }
 
+/*
+ * Second workload on the same fused-MLP family: the MLPs LAKE
+ * ports for load balancing (MLLB, §7.3, Fig. 10) and readahead classification
+ * (KML, §7.4, Fig. 11). PAPER.md gives no layer shapes or activations for
+ * either; the shapes are readings (R23-R26) and this function takes them as
+ * arguments. Plain definition, per input row i:
+ *   h = x[i]
+ *   for each hidden layer l: per output j, acc = +0.0f, acc = fmaf(h[k], W_l[j][k], acc)
+ *       for k ascending, z = acc + b_l[j] (one rounding), then
+ *       act 0 (ReLU):    h'[j] = (z > 0.0f) ? z : +0.0f          (R15, as for LinnOS)
+ *       act 1 (sigmoid): h'[j] = 1.0f / (1.0f + expf(-z))        (R25)
+ *   output layer (identity): out[c] = acc_c + b_out[c], c < C = widths[n_layers]
+ *   class = the first c with out[c] maximal: best = 0; for c = 1..C-1, best = c when
+ *           out[c] > out[best]  (R26; for C = 2 this is R14's decision; NaN never wins)
+ * blob: per layer W_l[widths[l+1]][widths[l]] row-major then b_l[widths[l+1]].
+ * x: float[n][widths[0]]; out: float[n][C] (may be NULL); cls: int32[n].
+ */
+int oracle_mlp_family(int n_layers, const int *widths, int act, const float *blob,
+                      const float *x, int64_t n, float *out, int32_t *cls, int nthreads)
+{
+    if (n_layers < 1 || (act != 0 && act != 1) || widths[n_layers] < 2) return 1;
+    int maxw = 0;
+    for (int l = 0; l <= n_layers; ++l) {
+        if (widths[l] <= 0) return 1;
+        if (widths[l] > maxw) maxw = widths[l];
+    }
+    const int C = widths[n_layers];
+#ifdef _OPENMP
+    const int nt = nthreads > 0 ? nthreads : omp_get_num_procs();
+#else
+    (void)nthreads;
+#endif
+#pragma omp parallel for schedule(static) num_threads(nt)
+    for (int64_t i = 0; i < n; ++i) {
+        float bufa[maxw], bufb[maxw];
+        float *h = bufa, *hn = bufb;
+        memcpy(h, x + i * widths[0], sizeof(float) * (size_t)widths[0]);
+        const float *p = blob;
+        for (int l = 0; l < n_layers; ++l) {
+            const int K = widths[l], N = widths[l + 1];
+            const float *W = p;
+            const float *b = p + (int64_t)N * K;
+            p = b + N;
+            const int hidden = (l + 1 < n_layers);
+            for (int j = 0; j < N; ++j) {
+                float acc = +0.0f;
+                for (int k = 0; k < K; ++k) acc = fmaf(h[k], W[(int64_t)j * K + k], acc);
+                float z = acc + b[j];
+                if (!hidden) hn[j] = z;
+                else if (act == 0) hn[j] = (z > 0.0f) ? z : 0.0f;
+                else hn[j] = 1.0f / (1.0f + expf(-z));
+            }
+            float *t = h; h = hn; hn = t;
+        }
+        int best = 0;
+        for (int c = 1; c < C; ++c)
+            if (h[c] > h[best]) best = c;
+        cls[i] = best;
+        if (out) memcpy(out + i * C, h, sizeof(float) * (size_t)C);
+    }
+    return 0;
+}
+
 int oracle_max_threads(void)
 {
 #ifdef _OPENMP
