@@ -53,7 +53,7 @@ def parse():
     p.add_argument("--prec", default=None, choices=["fp32", "f16", "bf16"])
     p.add_argument("--arch", type=int, default=None)
     p.add_argument("--n-ios", dest="n", type=int, default=None)
-    p.add_argument("--mode", default="throughput", choices=["throughput", "sweep", "report"])
+    p.add_argument("--mode", default="throughput", choices=["throughput", "sweep", "report", "family"])
     p.add_argument("--sweep-out", default=None)
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu", action="store_true")
@@ -674,6 +674,127 @@ def run_report(args):
     print(json.dumps({"metric": "C3/C4/C5 report", "rows": len(rows)}))
 
 
+# ------------------------------------------------------------------ NEXT-4 MLP family
+FP32_PEAK_TFLOPS = 74.4  # 148 SM x 128 FP32 lanes x 2 FLOP x 1.965 GHz
+
+
+def run_family(args):
+    """NEXT-4: the MLLB / KML-shaped MLPs (include/lake_mlp.h, readings
+    R23-R26). Per model: batch latency vs batch size 1..1024 (Fig. 10 / Fig. 11's range,
+    P:1436-1535): end to end through the public call with host buffers (pinned H2D of the
+    features, lake_mlp_infer, D2H of the classes, sync; host clock) and device-only (CUDA
+    events), beside the 1-thread oracle for the same batch, with the crossover batch; then
+    throughput at 2^24 rows (inputs resident in HBM, larger than L2) against the FP32 and
+    HBM rooflines, and the oracle on all host cores on a bounded sample."""
+    import torch
+    import oracle
+    from paper_conf_asplos_finglertyshar23_b200 import lake
+    from paper_conf_asplos_finglertyshar23_b200.inputs import family
+    torch.cuda.set_device(0)
+    dev = torch.device("cuda", 0)
+    stream = torch.cuda.current_stream()
+    pk = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    peaks = json.load(open(pk)) if os.path.exists(pk) else {}
+    hbm_peak = float(peaks.get("hbm_gbs", 7700.0))
+    hbm_src = "measured (MEASURED_PEAKS.json hbm_gbs)" if "hbm_gbs" in peaks else "nominal fallback"
+    rows = []
+    for mid, (name, cfg) in enumerate(sorted(family.FAMILY.items())):
+        widths, act = cfg["widths"], cfg["act"]
+        blob = family.weights(widths, 0)
+        lake.mlp_load(mid, widths, act, blob, 0)
+        C = widths[-1]
+        x_all = family.features(1 << 24, widths[0], 3000 + mid)
+        cross = None
+        for b in [1 << k for k in range(11)]:
+            x = np.ascontiguousarray(x_all[:b])
+            h_x = torch.from_numpy(x).pin_memory()
+            h_c = torch.empty(b, dtype=torch.int32).pin_memory()
+            d_x = torch.empty_like(h_x, device=dev)
+            d_c = torch.empty(b, dtype=torch.int32, device=dev)
+            reps, warm = 200, 20
+
+            def once():
+                d_x.copy_(h_x, non_blocking=True)
+                lake.mlp_infer(d_x, b, mid, d_c, None, stream)
+                h_c.copy_(d_c, non_blocking=True)
+                stream.synchronize()
+            for _ in range(warm):
+                once()
+            ts = []
+            for _ in range(reps):
+                t0 = time.perf_counter()
+                once()
+                ts.append((time.perf_counter() - t0) * 1e6)
+            ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            ev0.record(stream)
+            for _ in range(reps):
+                lake.mlp_infer(d_x, b, mid, d_c, None, stream)
+            ev1.record(stream)
+            torch.cuda.synchronize()
+            dev_us = ev0.elapsed_time(ev1) * 1e3 / reps
+            _, rc = oracle.mlp_family(widths, act, blob, x, nthreads=1)
+            if not np.array_equal(h_c.numpy(), rc) and act == family.ACT_RELU:
+                raise RuntimeError(f"{name} b={b}: classes differ from the oracle")
+            oreps = max(1, min(200, int(2e5 / b)))
+            t0 = time.perf_counter()
+            for _ in range(oreps):
+                oracle.mlp_family(widths, act, blob, x, nthreads=1)
+            cpu_us = (time.perf_counter() - t0) * 1e6 / oreps
+            med = float(np.median(ts))
+            if cross is None and med < cpu_us:
+                cross = b
+            row = dict(model=name, widths=list(widths), act=["relu", "sigmoid"][act], batch=b,
+                       e2e_us_median=round(med, 2), e2e_us_p99=round(float(np.percentile(ts, 99)), 2),
+                       device_us=round(dev_us, 2), cpu_1thread_us=round(cpu_us, 2))
+            rows.append(row)
+            log(json.dumps(row))
+        # throughput at 2^24 rows
+        n = 1 << 24
+        d_x = torch.from_numpy(x_all).to(dev)
+        d_c = torch.empty(n, dtype=torch.int32, device=dev)
+        for _ in range(max(3, args.warmup)):
+            lake.mlp_infer(d_x, n, mid, d_c, None, stream)
+        K = max(5, args.steps)
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ev0.record(stream)
+        for _ in range(K):
+            lake.mlp_infer(d_x, n, mid, d_c, None, stream)
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        ms = ev0.elapsed_time(ev1) / K
+        fma = sum(widths[l] * widths[l + 1] for l in range(len(widths) - 1))
+        byt = 4 * widths[0] + 4
+        tflops = n * 2 * fma / (ms * 1e-3) / 1e12
+        gbps = n * byt / (ms * 1e-3) / 1e9
+        samp = np.arange(0, n, 64)
+        t0 = time.perf_counter()
+        oracle.mlp_family(widths, act, blob, x_all[samp], nthreads=0)
+        cpu_s = time.perf_counter() - t0
+        row = dict(model=name, widths=list(widths), act=["relu", "sigmoid"][act], n_rows=n,
+                   kernel_ms=round(ms, 4), rows_per_s=round(n / (ms * 1e-3), 1),
+                   flop_per_row=2 * fma, bytes_per_row=byt,
+                   roofline_alu={"achieved": round(tflops, 2), "peak": FP32_PEAK_TFLOPS,
+                                 "unit": "TFLOP/s", "frac": round(tflops / FP32_PEAK_TFLOPS, 4),
+                                 "peak_source": "derived from unit counts (DESIGN.md §7.1)"},
+                   roofline_hbm={"achieved": round(gbps, 1), "peak": hbm_peak, "unit": "GB/s",
+                                 "frac": round(gbps / hbm_peak, 4), "peak_source": hbm_src},
+                   cpu_baseline={"value": round(len(samp) / cpu_s, 1), "unit": "rows/s",
+                                 "cores": oracle.max_threads(), "kind": "oracle",
+                                 "sample": f"stride-64 sample of {len(samp)} rows"})
+        rows.append(row)
+        log(json.dumps(row))
+        rows.append(dict(model=name, crossover_batch=cross))
+        lake.mlp_unload(mid, 0)
+        del d_x, d_c
+    path = args.sweep_out or os.path.join(ROOT, "gpurun_out", "family.jsonl")
+    os.makedirs(os.path.dirname(path), exist_ok=True)
+    with open(path, "w") as f:
+        for r in rows:
+            f.write(json.dumps(r) + "\n")
+    print(json.dumps({"metric": "NEXT-4 MLP family: latency vs batch, throughput", "rows": len(rows),
+                      "crossovers": [r for r in rows if "crossover_batch" in r]}))
+
+
 def main():
     args = parse()
     if args.impl == "reference":
@@ -682,6 +803,8 @@ def main():
         run_sweep(args)
     elif args.mode == "report":
         run_report(args)
+    elif args.mode == "family":
+        run_family(args)
     else:
         run_ours(args)
 

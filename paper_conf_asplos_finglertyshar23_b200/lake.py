@@ -42,6 +42,13 @@ EXPORTS = (
     "lake_linnos_auto_threshold", "lake_linnos_set_auto_threshold",
     "lake_linnos_server_start", "lake_linnos_server_infer", "lake_linnos_server_stop",
 )
+# every symbol include/lake_mlp.h declares (NEXT-4 MLP family)
+MLP_EXPORTS = (
+    "lake_mlp_blob_floats", "lake_mlp_load", "lake_mlp_unload", "lake_mlp_infer",
+    "lake_mlp_model_shape", "lake_mlp_force_generic",
+)
+LAKE_ACT_RELU, LAKE_ACT_SIGMOID = 0, 1
+LAKE_MLP_MAX_LAYERS, LAKE_MLP_MAX_WIDTH, LAKE_MLP_MAX_MODELS = 4, 64, 256
 
 
 class LakeError(RuntimeError):
@@ -88,6 +95,12 @@ def lib():
             "lake_linnos_server_start": (ctypes.c_int, [I32, P]),
             "lake_linnos_server_infer": (ctypes.c_int, [P, P, I32, P, P]),
             "lake_linnos_server_stop": (ctypes.c_int, [P]),
+            "lake_mlp_blob_floats": (SZ, [I32, P]),
+            "lake_mlp_load": (ctypes.c_int, [I32, I32, P, I32, P, SZ, I32]),
+            "lake_mlp_unload": (ctypes.c_int, [I32, I32]),
+            "lake_mlp_infer": (ctypes.c_int, [P, I64, I32, P, P, P]),
+            "lake_mlp_model_shape": (ctypes.c_int, [I32, I32, P, P, P]),
+            "lake_mlp_force_generic": (ctypes.c_int, [I32]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -258,3 +271,39 @@ class Server:
 
     def __exit__(self, *a):
         self.stop()
+
+
+# ---------------------------------------------------------------- NEXT-4 MLP family
+def mlp_blob_floats(widths) -> int:
+    w = np.ascontiguousarray(widths, dtype=np.int32)
+    return int(lib().lake_mlp_blob_floats(len(w) - 1, w.ctypes.data))
+
+
+def mlp_load(model_id: int, widths, act: int, blob: np.ndarray, device: int) -> None:
+    w = np.ascontiguousarray(widths, dtype=np.int32)
+    blob = np.ascontiguousarray(blob, dtype=np.float32)
+    _check(lib().lake_mlp_load(model_id, len(w) - 1, w.ctypes.data, act, blob.ctypes.data,
+                               blob.size, device), "mlp_load")
+
+
+def mlp_unload(model_id: int, device: int) -> None:
+    _check(lib().lake_mlp_unload(model_id, device), "mlp_unload")
+
+
+def mlp_infer(x, n: int, model_id: int, classes, out=None, stream=None) -> None:
+    _check(lib().lake_mlp_infer(_ptr(x), n, model_id, _ptr(classes), _ptr(out),
+                                _stream(stream)), "mlp_infer")
+
+
+def mlp_model_shape(model_id: int, device: int):
+    nl = ctypes.c_int32(0)
+    act = ctypes.c_int32(-1)
+    w = np.zeros(LAKE_MLP_MAX_LAYERS + 1, dtype=np.int32)
+    _check(lib().lake_mlp_model_shape(model_id, device, ctypes.byref(nl), w.ctypes.data,
+                                      ctypes.byref(act)), "mlp_model_shape")
+    return tuple(int(v) for v in w[: nl.value + 1]), act.value
+
+
+def mlp_force_generic(enable: bool) -> bool:
+    """Route every MLP-family model through the generic kernel; returns the previous value."""
+    return bool(lib().lake_mlp_force_generic(1 if enable else 0))

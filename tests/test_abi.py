@@ -13,23 +13,33 @@ from paper_conf_asplos_finglertyshar23_b200 import inputs, lake
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-def _declared():
-    src = open(os.path.join(ROOT, "include", "lake_linnos.h")).read()
+def _declared(header="lake_linnos.h", prefix="lake_linnos_"):
+    src = open(os.path.join(ROOT, "include", header)).read()
     src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
-    return sorted(set(re.findall(r"\b(lake_linnos_\w+)\s*\(", src)))
+    return sorted(set(re.findall(r"\b(" + prefix + r"\w+)\s*\(", src)))
+
+
+def _all_declared():
+    names = []
+    for h in sorted(os.listdir(os.path.join(ROOT, "include"))):
+        if h.endswith(".h"):
+            names += _declared(h, "lake_")
+    return sorted(set(names))
 
 
 def test_header_matches_binding_list():
     assert _declared() == sorted(lake.EXPORTS)
+    assert _declared("lake_mlp.h", "lake_mlp_") == sorted(lake.MLP_EXPORTS)
+    assert _all_declared() == sorted(lake.EXPORTS + lake.MLP_EXPORTS)
 
 
 def test_library_exports_every_declared_symbol():
     L = lake.lib()
-    for name in _declared():
+    for name in _all_declared():
         assert hasattr(L, name), name
     # the binding resolves by the same names
     dl = ctypes.CDLL(lake.LIB_PATH)
-    for name in _declared():
+    for name in _all_declared():
         getattr(dl, name)
 
 
@@ -101,3 +111,35 @@ def test_auto_thresholds_roundtrip():
         lake.set_auto_threshold(5, 1)
     with pytest.raises(lake.LakeError):
         lake.set_auto_threshold(0, -1)
+
+
+def test_mlp_family_host_validation():
+    """NEXT-4 ABI (include/lake_mlp.h): shape / argument errors answer on the host."""
+    from paper_conf_asplos_finglertyshar23_b200.inputs import family
+    L = lake.lib()
+    for name, cfg in family.FAMILY.items():
+        assert lake.mlp_blob_floats(cfg["widths"]) == family.blob_floats(cfg["widths"])
+    assert lake.mlp_blob_floats([15, 10, 10, 2]) == 15 * 10 + 10 + 10 * 10 + 10 + 10 * 2 + 2
+    assert lake.mlp_blob_floats([5, 15, 15, 4]) == 5 * 15 + 15 + 15 * 15 + 15 + 15 * 4 + 4
+    for bad in ([3, 1], [0, 4, 2], [3, 65, 2], [3, 4, 4, 4, 4, 2], [3]):
+        assert lake.mlp_blob_floats(bad) == 0, bad
+    w = np.array([5, 15, 15, 4], np.int32)
+    blob = family.weights(w, 0)
+    P = w.ctypes.data
+    assert L.lake_mlp_load(-1, 3, P, 1, blob.ctypes.data, blob.size, 0) == lake.LAKE_ERR_INVAL
+    assert L.lake_mlp_load(256, 3, P, 1, blob.ctypes.data, blob.size, 0) == lake.LAKE_ERR_INVAL
+    assert L.lake_mlp_load(0, 3, P, 2, blob.ctypes.data, blob.size, 0) == lake.LAKE_ERR_INVAL
+    assert L.lake_mlp_load(0, 3, P, 1, blob.ctypes.data, blob.size - 1, 0) == lake.LAKE_ERR_INVAL
+    assert L.lake_mlp_load(0, 3, P, 1, None, blob.size, 0) == lake.LAKE_ERR_INVAL
+    bad = blob.copy()
+    bad[7] = np.inf
+    assert L.lake_mlp_load(0, 3, P, 1, bad.ctypes.data, bad.size, 0) == lake.LAKE_ERR_INVAL
+    assert L.lake_mlp_load(0, 3, P, 1, blob.ctypes.data, blob.size, -1) == lake.LAKE_ERR_INVAL
+    assert L.lake_mlp_infer(None, -1, 0, None, None, None) == lake.LAKE_ERR_INVAL
+    assert L.lake_mlp_infer(None, 0, 0, None, None, None) == lake.LAKE_OK      # n == 0: no-op
+    assert L.lake_mlp_infer(None, 10, 0, None, None, None) == lake.LAKE_ERR_INVAL
+    assert L.lake_mlp_infer(16, 10, 0, 18, None, None) == lake.LAKE_ERR_INVAL  # misaligned
+    assert L.lake_mlp_infer(16, 2 ** 31, 0, 32, None, None) == lake.LAKE_ERR_INVAL
+    assert L.lake_mlp_unload(-1, 0) == lake.LAKE_ERR_INVAL
+    assert L.lake_mlp_unload(5, 0) == lake.LAKE_ERR_NOMODEL
+    assert L.lake_mlp_model_shape(5, 0, None, None, None) == lake.LAKE_ERR_INVAL
