@@ -680,7 +680,7 @@ FP32_PEAK_TFLOPS = 74.4  # 148 SM x 128 FP32 lanes x 2 FLOP x 1.965 GHz (DESIGN.
 
 def run_family(args):
     """NEXT-4: the MLLB / KML-shaped MLPs (include/lake_mlp.h, readings
-    R23-R26). Per model: batch latency vs batch size 1..1024 (Fig. 10 / Fig. 11's range,
+    R25-R28). Per model: batch latency vs batch size 1..1024 (Fig. 10 / Fig. 11's range,
     P:1436-1535): end to end through the public call with host buffers (pinned H2D of the
     features, lake_mlp_infer, D2H of the classes, sync; host clock) and device-only (CUDA
     events), beside the 1-thread oracle for the same batch, with the crossover batch; then

@@ -13,7 +13,7 @@
  *   - batch scoring is the feature registry's score_features (Table 1).
  *
  * PAPER.md gives neither model's layer widths, activation or features, so this ABI takes
- * them as arguments; the shapes the tests and the bench use are readings R23-R26 in
+ * them as arguments; the shapes the tests and the bench use are readings R25-R28 in
  * DESIGN.md §3 (MLLB 15->10->10->2 ReLU, KML 5->15->15->4 sigmoid).
  *
  * Conventions (status codes, devices, streams, ownership, asynchrony, determinism) are
@@ -46,7 +46,7 @@ extern "C" {
 /* Hidden-layer activation; the output layer is always the identity. */
 enum lake_mlp_act {
     LAKE_ACT_RELU = 0,    /* h = (z > 0.0f) ? z : +0.0f                          (R15) */
-    LAKE_ACT_SIGMOID = 1  /* h = 1.0f / (1.0f + expf(-z)), IEEE division, full expf (R25) */
+    LAKE_ACT_SIGMOID = 1  /* h = 1.0f / (1.0f + expf(-z)), IEEE division, full expf (R27) */
 };
 
 /* Exact blob length in floats for a shape, or 0 if the shape is invalid:
@@ -88,7 +88,7 @@ int lake_mlp_model_shape(int32_t model_id, int32_t device, int32_t *n_layers_out
                          int32_t *widths_out, int32_t *act_out);
 
 /* Kernel selection. Shapes with a compile-time-specialised kernel (the MLLB and KML
- * readings, R23/R24) use it by default; enable != 0 routes every model through the generic
+ * readings, R25/R26) use it by default; enable != 0 routes every model through the generic
  * runtime-shape kernel instead (process-wide; both kernels compute the same values — the
  * parity tests run both). Returns the previous setting (0 or 1). */
 int lake_mlp_force_generic(int32_t enable);

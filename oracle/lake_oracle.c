@@ -284,16 +284,16 @@ void oracle_capture_rows(const int64_t *a, const int64_t *c, const int32_t *dev,
  * Second workload on the same fused-MLP family: the MLPs LAKE
  * ports for load balancing (MLLB, §7.3, Fig. 10) and readahead classification
  * (KML, §7.4, Fig. 11). PAPER.md gives no layer shapes or activations for
- * either; the shapes are readings (R23-R26) and this function takes them as
+ * either; the shapes are readings (R25-R28) and this function takes them as
  * arguments. Plain definition, per input row i:
  *   h = x[i]
  *   for each hidden layer l: per output j, acc = +0.0f, acc = fmaf(h[k], W_l[j][k], acc)
  *       for k ascending, z = acc + b_l[j] (one rounding), then
  *       act 0 (ReLU):    h'[j] = (z > 0.0f) ? z : +0.0f          (R15, as for LinnOS)
- *       act 1 (sigmoid): h'[j] = 1.0f / (1.0f + expf(-z))        (R25)
+ *       act 1 (sigmoid): h'[j] = 1.0f / (1.0f + expf(-z))        (R27)
  *   output layer (identity): out[c] = acc_c + b_out[c], c < C = widths[n_layers]
  *   class = the first c with out[c] maximal: best = 0; for c = 1..C-1, best = c when
- *           out[c] > out[best]  (R26; for C = 2 this is R14's decision; NaN never wins)
+ *           out[c] > out[best]  (R28; for C = 2 this is R14's decision; NaN never wins)
  * blob: per layer W_l[widths[l+1]][widths[l]] row-major then b_l[widths[l+1]].
  * x: float[n][widths[0]]; out: float[n][C] (may be NULL); cls: int32[n].
  */

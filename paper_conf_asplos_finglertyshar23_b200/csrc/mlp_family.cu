@@ -165,7 +165,7 @@ struct GenericBody {
   }
 };
 
-// Fixed shapes (the two readings the bench runs, R23/R24): widths, offsets and activation
+// Fixed shapes (the two readings the bench runs, R25/R26): widths, offsets and activation
 // are compile-time, the whole network is unrolled with every activation in registers, the
 // weights are read as LDS.128 broadcasts of W[j][k..k+3] (row-major, K padded to 4; the pad
 // is never read) and each weight feeds RPT rows. Same operation order as the oracle.
@@ -491,7 +491,7 @@ int lake_mlp_load(int32_t model_id, int32_t n_layers, const int32_t *widths, int
     q += N;
   }
 
-  // compile-time-shape image for the two shapes with a specialised kernel (R23/R24)
+  // compile-time-shape image for the two shapes with a specialised kernel (R25/R26)
   std::vector<float> fx;
   if (shape_is<MllbShape>(m)) {
     m.fixed = 1;

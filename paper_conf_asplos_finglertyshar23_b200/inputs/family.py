@@ -2,7 +2,7 @@
 
 Holds none of the method's arithmetic: it draws feature rows and random-init weights.
 PAPER.md gives neither the shapes nor the features of these models (§7.3 P:1471-1475,
-§7.4); the shapes are readings R23-R26:
+§7.4); the shapes are readings R25-R28:
 
 * ``mllb``: 15 per-task load-balancing features -> 10 -> 10 -> 2 (migrate / stay), ReLU.
 * ``kml``:  5 per-process I/O-pattern features -> 15 -> 15 -> 4 readahead classes, sigmoid.

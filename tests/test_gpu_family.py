@@ -3,7 +3,7 @@
 ReLU models: outputs and classes bit-exact (same operation order, R15).
 Sigmoid models: the kernel's expf / IEEE division and glibc's expf differ by a few ulp,
 so outputs are compared within 1e-5 relative (S19 form: |d| / max(|ref|, rms(ref))) and
-classes must agree wherever the oracle's top-two margin exceeds 1e-4 (R25/R26).
+classes must agree wherever the oracle's top-two margin exceeds 1e-4 (R27/R28).
 Inputs come from the seeded generators; expected values only from oracle/."""
 import numpy as np
 import pytest

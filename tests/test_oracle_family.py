@@ -1,4 +1,4 @@
-"""Pins for the oracle's NEXT-4 MLP family (oracle.mlp_family; readings R23-R26).
+"""Pins for the oracle's NEXT-4 MLP family (oracle.mlp_family; readings R25-R28).
 
 Each test checks the oracle against something other than itself:
 * hand-worked examples (tests/golden/family_examples.txt): sigma(0) = 0.5, saturation,
