@@ -290,9 +290,20 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
 
 #ifdef LAKE_TRACE
   unsigned long long *const tr_buf = g_lake_trace;  // read once: events cost no global load
+#ifdef LAKE_TRACE_QUAD  // streams: epilogue warps 4, 5, 6, 3 of rank 0 (TMEM quadrants 0-3)
+  const int tr_stream = !(tr_buf && cid == 0 && rank == 0) || lane != 0 ? -1
+                      : (warp >= kWarpEpi && warp < kWarpEpi + 4) ? (int)((warp - kWarpEpi + 3) & 3) : -1;
+#elif defined(LAKE_TRACE_PAIR)  // streams: MMA, epilogue warp 3 of rank 0 / rank 1, warp 7 of rank 0
+  const int tr_stream = !(tr_buf && cid == 0) || lane != 0 ? -1
+                      : (warp == kWarpMma && rank == 0) ? 0
+                      : (warp == kWarpEpi && rank == 0) ? 1
+                      : (warp == kWarpEpi && rank == 1) ? 2
+                      : (warp == kWarpEpi + 4 && rank == 0) ? 3 : -1;
+#else
   const int tr_stream = !(tr_buf && cid == 0 && rank == 0) ? -1
                       : (warp == kWarpMma && lane == 0) ? 0 : (warp == kWarpEpi && lane == 0) ? 1
                       : (warp == kWarpMma - 1 && lane == 0) ? 2 : (threadIdx.x == 0) ? 3 : -1;
+#endif
   uint32_t tr_i = 0;
 #endif
   const int64_t n_tiles = ts.n_tiles_dev ? (int64_t)*ts.n_tiles_dev : ts.n_tiles;

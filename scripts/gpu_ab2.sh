@@ -1,0 +1,15 @@
+#!/bin/bash
+# A/B (twice, interleaved) the kernel variants under build/var/*: parity subset + C5 bench
+mkdir -p gpurun_out
+out=gpurun_out/ab_${1:-x}.txt
+: > $out
+for rep in 1 2; do
+for v in build/var/*/; do
+  name=$(basename $v)
+  export LAKE_LINNOS_LIB=$v/liblake_linnos.so
+  t=""
+  if [ $rep = 1 ]; then t=$(timeout 300 python -m pytest tests/test_gpu_parity.py -m gpu -q -x -p no:cacheprovider 2>&1 | tail -1); fi
+  b=$(timeout 200 python bench.py --steps 10 --warmup 3 --no-cpu --no-e2e 2>/dev/null | python -c "import json,sys; d=json.loads(sys.stdin.read()); r=d['roofline']; print(f\"{d['value']/1e9:.3f} Ginf/s kernel {r['kernel_ms']:.3f} ms frac {r['frac']:.4f}\")")
+  echo "$name | $t | $b" >> $out
+done
+done

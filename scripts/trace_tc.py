@@ -15,7 +15,7 @@ from paper_conf_asplos_finglertyshar23_b200 import inputs, lake  # noqa: E402
 KIND = {1: "XFULL", 2: "TEMPTY", 3: "HREADY", 4: "COMMIT", 5: "DFULL", 6: "CHUNK",
         7: "LAYEREND", 8: "XEMPTY", 9: "XARRIVE", 10: "ISSUED", 11: "LDWAIT", 12: "STS",
         13: "FENCE"}
-STREAM = {0: "mma", 1: "epi4", 2: "epi11", 3: "dig"}
+STREAM = ({0: "mma", 1: "e3r1", 2: "e3r2", 3: "e7r1"} if os.environ.get("LAKE_TRACE_PAIR") else {0: "q0w4", 1: "q1w5", 2: "q2w6", 3: "q3w3"} if os.environ.get("LAKE_TRACE_QUAD") else {0: "mma", 1: "epi4", 2: "epi11", 3: "dig"})
 CAP = 1 << 16
 
 cfg = sys.argv[1] if len(sys.argv) > 1 else "C5"
@@ -50,7 +50,7 @@ rows.sort()
 clk = np.array([r[0] for r in rows])
 tiles = max(r[3] for r in rows) + 1
 print(f"events {len(rows)}, tiles in cluster 0: {tiles}, span {clk[-1] - clk[0]} cycles, {(clk[-1] - clk[0]) / tiles:.0f} cycles/tile")
-c0 = np.array([r[0] for r in rows if r[2] == 4 and r[4] == 0])
+c0 = np.array([r[0] for r in rows if (r[2] == 4 and r[4] == 0) or (r[2] == 5 and r[4] == 0 and r[1] == 0)])
 d = np.diff(np.sort(c0))
 print(f"tile period (L0 commits): median {np.median(d):.0f} p10 {np.percentile(d, 10):.0f} p90 {np.percentile(d, 90):.0f}")
 mid = tiles // 2
