@@ -90,7 +90,11 @@ enum lake_arch {
     LAKE_ARCH_NN2 = 2  /* 31 -> 256 -> 256 -> 256 -> 2  */
 };
 
-/* flags for lake_linnos_infer*: bit 0 = input kind, bits 4..6 = precision path. */
+/* flags for lake_linnos_infer*: bit 0 = input kind, bits 4..6 = precision path, bits 8..9 =
+ * element type of the per-I/O model ids (infer_multi / infer_host; ignored by calls that
+ * take no ids). Narrow ids cut the host->device bytes of the host-buffer path (PCIe-bound,
+ * DESIGN.md §7): 64 per-SSD models fit in one byte. An id the type cannot hold a loaded model
+ * for is simply unknown (decision 0, NaN logits). */
 enum lake_flags {
     LAKE_IN_DIGITS  = 0x00, /* in = const uint8_t[n][32] (pad byte must be 0)           */
     LAKE_IN_RAW     = 0x01, /* in = const lake_io_raw_t[n]; digitised inside the kernel  */
@@ -100,8 +104,12 @@ enum lake_flags {
     LAKE_PREC_BF16  = 0x20, /* tcgen05 tensor cores, bf16 operands, fp32 accumulation     */
     LAKE_PREC_TF32  = 0x30, /* reserved: returns LAKE_ERR_UNSUPPORTED (SMEM)   */
     LAKE_PREC_AUTO  = 0x70, /* FP32 below the model's AUTO threshold, else F16 (below)   */
+    LAKE_IDS_I32    = 0x000, /* model_ids: int32_t[n] (default)                         */
+    LAKE_IDS_U16    = 0x100, /* model_ids: uint16_t[n]                                   */
+    LAKE_IDS_U8     = 0x200, /* model_ids: uint8_t[n]                                    */
     LAKE_IN_MASK    = 0x01,
-    LAKE_PREC_MASK  = 0x70
+    LAKE_PREC_MASK  = 0x70,
+    LAKE_IDS_MASK   = 0x300
 };
 /* LAKE_PREC_AUTO (the paper's profitability policy, §4.2 P:583-603 and
  * Fig. 3, restricted to GPU paths since there is no CPU fallback): a call with n

@@ -242,8 +242,12 @@ int64_t auto_min(int32_t arch) {
   return g_auto_min[arch].load();
 }
 
+int id_kind_of(uint32_t flags) { return (int)((flags & LAKE_IDS_MASK) >> 8); }
+size_t id_bytes_of(uint32_t flags) { return (size_t)4 >> id_kind_of(flags); }
+
 int check_flags(uint32_t flags, int64_t n, int *in_kind, int *prec, int32_t arch = -1) {
-  if (flags & ~(uint32_t)(LAKE_IN_MASK | LAKE_PREC_MASK)) return LAKE_ERR_INVAL;
+  if (flags & ~(uint32_t)(LAKE_IN_MASK | LAKE_PREC_MASK | LAKE_IDS_MASK)) return LAKE_ERR_INVAL;
+  if ((flags & LAKE_IDS_MASK) == LAKE_IDS_MASK) return LAKE_ERR_INVAL;
   *in_kind = (int)(flags & LAKE_IN_MASK);
   const uint32_t p = flags & LAKE_PREC_MASK;
   switch (p) {
@@ -480,8 +484,16 @@ size_t lake_linnos_workspace_bytes(int64_t n) {
   return group_workspace_bytes(n);
 }
 
+int multi_group_impl(int64_t n, const void *model_ids, int id_kind, void *workspace,
+                     size_t ws_bytes, void *stream);
+
 int lake_linnos_multi_group(int64_t n, const int32_t *model_ids, void *workspace,
                             size_t ws_bytes, void *stream) {
+  return multi_group_impl(n, model_ids, 0, workspace, ws_bytes, stream);
+}
+
+int multi_group_impl(int64_t n, const void *model_ids, int id_kind, void *workspace,
+                     size_t ws_bytes, void *stream) {
   if (n < 0 || n > (int64_t)INT32_MAX) return LAKE_ERR_INVAL;
   if (n > 0 && !model_ids) return LAKE_ERR_INVAL;
   if (!workspace) return LAKE_ERR_INVAL;
@@ -500,7 +512,7 @@ int lake_linnos_multi_group(int64_t n, const int32_t *model_ids, void *workspace
     table = st->table;
   }
   return cuda_status(
-      launch_group(n, model_ids, table, workspace, 0, static_cast<cudaStream_t>(stream)));
+      launch_group(n, model_ids, id_kind, table, workspace, 0, static_cast<cudaStream_t>(stream)));
 }
 
 int lake_linnos_multi_grouped(const void *in, uint32_t flags, int64_t n, uint8_t *decisions,
@@ -537,9 +549,10 @@ int lake_linnos_infer_multi(const void *in, uint32_t flags, int64_t n, const int
   if (n == 0) return LAKE_OK;
   if (!in || !decisions || !model_ids || !workspace) return LAKE_ERR_INVAL;
   if (check_input_ptr(in, in_kind) != LAKE_OK) return LAKE_ERR_INVAL;
-  rc = lake_linnos_multi_group(n, model_ids, workspace, ws_bytes, stream);
+  rc = multi_group_impl(n, model_ids, id_kind_of(flags), workspace, ws_bytes, stream);
   if (rc != LAKE_OK) return rc;
-  return lake_linnos_multi_grouped(in, flags, n, decisions, logits, workspace, ws_bytes, stream);
+  return lake_linnos_multi_grouped(in, flags & ~(uint32_t)LAKE_IDS_MASK, n, decisions, logits,
+                                   workspace, ws_bytes, stream);
 }
 
 int lake_linnos_multi_status(const void *workspace, size_t ws_bytes, int64_t *n_unknown,
@@ -657,6 +670,7 @@ int lake_linnos_infer_host(const void *h_in, uint32_t flags, int64_t n, int32_t 
   }
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   const size_t in_b = in_kind == LAKE_IN_RAW ? 36 : 32;
+  const size_t id_b = id_bytes_of(flags);
   const int64_t chunk = n < kHostChunk ? n : kHostChunk;
   const SlotLayout L = slot_layout(chunk, in_b);
   const int64_t nchunks = (n + chunk - 1) / chunk;
@@ -684,7 +698,7 @@ int lake_linnos_infer_host(const void *h_in, uint32_t flags, int64_t n, int32_t 
     // one chunk: nothing to overlap, so stay on the caller's stream (no cross-stream hops)
     cudaError_t e = cudaMemcpyAsync(base + L.in, h_in, n * in_b, cudaMemcpyHostToDevice, s);
     if (e == cudaSuccess && h_model_ids)
-      e = cudaMemcpyAsync(base + L.ids, h_model_ids, n * 4, cudaMemcpyHostToDevice, s);
+      e = cudaMemcpyAsync(base + L.ids, h_model_ids, n * id_b, cudaMemcpyHostToDevice, s);
     if (e != cudaSuccess) return cuda_status(e);
     uint8_t *d_dec = base + L.dec;
     float *d_log = h_logits ? reinterpret_cast<float *>(base + L.log) : nullptr;
@@ -717,7 +731,8 @@ int lake_linnos_infer_host(const void *h_in, uint32_t flags, int64_t n, int32_t 
       e = cudaMemcpyAsync(sb + L.in, static_cast<const uint8_t *>(h_in) + off * in_b, cn * in_b,
                           cudaMemcpyHostToDevice, pp->h2d);
     if (e == cudaSuccess && h_model_ids)
-      e = cudaMemcpyAsync(sb + L.ids, h_model_ids + off, cn * 4, cudaMemcpyHostToDevice, pp->h2d);
+      e = cudaMemcpyAsync(sb + L.ids, reinterpret_cast<const uint8_t *>(h_model_ids) + off * id_b,
+                          cn * id_b, cudaMemcpyHostToDevice, pp->h2d);
     if (e == cudaSuccess) e = cudaEventRecord(pp->in_ready[slot], pp->h2d);
     if (e == cudaSuccess) e = cudaStreamWaitEvent(s, pp->in_ready[slot], 0);
     if (e == cudaSuccess && c >= 2) e = cudaStreamWaitEvent(s, pp->out_done[slot], 0);  // outputs read

@@ -63,8 +63,9 @@ __device__ __forceinline__ bool known(const DevModel *table, int32_t m) {
   return m >= 0 && m < LAKE_MAX_MODELS && table[m].arch >= 0;
 }
 
+template <typename IdT>
 __global__ void __launch_bounds__(kGBlock)
-group_hist(const int32_t *__restrict__ ids, int64_t n, const DevModel *__restrict__ table,
+group_hist(const IdT *__restrict__ ids, int64_t n, const DevModel *__restrict__ table,
            WsHeader *h) {
   __shared__ int32_t cnt[LAKE_MAX_MODELS + 1];
   for (int64_t base = (int64_t)blockIdx.x * kChunk; base < n; base += (int64_t)gridDim.x * kChunk) {
@@ -72,7 +73,7 @@ group_hist(const int32_t *__restrict__ ids, int64_t n, const DevModel *__restric
     __syncthreads();
     const int64_t end = (base + kChunk) < n ? base + kChunk : n;
     for (int64_t i = base + threadIdx.x; i < end; i += kGBlock) {
-      const int32_t m = __ldg(ids + i);
+      const int32_t m = (int32_t)__ldg(ids + i);
       atomicAdd(&cnt[known(table, m) ? m : LAKE_MAX_MODELS], 1);
     }
     __syncthreads();
@@ -136,8 +137,9 @@ group_scan(WsHeader *h) {
   }
 }
 
+template <typename IdT>
 __global__ void __launch_bounds__(kGBlock)
-group_scatter(const int32_t *__restrict__ ids, int64_t n, const DevModel *__restrict__ table,
+group_scatter(const IdT *__restrict__ ids, int64_t n, const DevModel *__restrict__ table,
               WsHeader *h, int32_t *__restrict__ perm) {
   __shared__ int32_t cnt[LAKE_MAX_MODELS + 1];
   __shared__ int32_t basep[LAKE_MAX_MODELS + 1];
@@ -146,7 +148,7 @@ group_scatter(const int32_t *__restrict__ ids, int64_t n, const DevModel *__rest
     __syncthreads();
     const int64_t end = (base + kChunk) < n ? base + kChunk : n;
     for (int64_t i = base + threadIdx.x; i < end; i += kGBlock) {
-      const int32_t m = __ldg(ids + i);
+      const int32_t m = (int32_t)__ldg(ids + i);
       atomicAdd(&cnt[known(table, m) ? m : LAKE_MAX_MODELS], 1);
     }
     __syncthreads();
@@ -157,7 +159,7 @@ group_scatter(const int32_t *__restrict__ ids, int64_t n, const DevModel *__rest
     }
     __syncthreads();
     for (int64_t i = base + threadIdx.x; i < end; i += kGBlock) {
-      const int32_t m0 = __ldg(ids + i);
+      const int32_t m0 = (int32_t)__ldg(ids + i);
       const int32_t m = known(table, m0) ? m0 : LAKE_MAX_MODELS;
       const int32_t r = atomicAdd(&cnt[m], 1);
       perm[basep[m] + r] = (int32_t)i;
@@ -260,8 +262,8 @@ static GroupPtrs group_ptrs(void *ws, int64_t n) {
   return p;
 }
 
-cudaError_t launch_group(int64_t n, const int32_t *model_ids, const DevModel *table, void *ws,
-                         int /*tile_rows*/, cudaStream_t s) {
+cudaError_t launch_group(int64_t n, const void *model_ids, int id_kind, const DevModel *table,
+                         void *ws, int /*tile_rows*/, cudaStream_t s) {
   GroupPtrs p = group_ptrs(ws, n);
   cudaError_t e = cudaMemsetAsync(p.h, 0, sizeof(WsHeader), s);
   if (e != cudaSuccess) return e;
@@ -270,9 +272,18 @@ cudaError_t launch_group(int64_t n, const int32_t *model_ids, const DevModel *ta
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   const int64_t chunks = (n + kChunk - 1) / kChunk;
   const int grid = (int)(chunks < 2 * sms ? chunks : 2 * sms);
-  if (grid > 0) group_hist<<<grid, kGBlock, 0, s>>>(model_ids, n, table, p.h);
+  auto hist = [&](auto *ids) {
+    if (grid > 0) group_hist<<<grid, kGBlock, 0, s>>>(ids, n, table, p.h);
+  };
+  auto scatter = [&](auto *ids) {
+    if (grid > 0) group_scatter<<<grid, kGBlock, 0, s>>>(ids, n, table, p.h, p.perm);
+  };
+  const int32_t *i32 = static_cast<const int32_t *>(model_ids);
+  const uint16_t *u16 = static_cast<const uint16_t *>(model_ids);
+  const uint8_t *u8 = static_cast<const uint8_t *>(model_ids);
+  if (id_kind == 1) hist(u16); else if (id_kind == 2) hist(u8); else hist(i32);
   group_scan<<<1, LAKE_MAX_MODELS, 0, s>>>(p.h);
-  if (grid > 0) group_scatter<<<grid, kGBlock, 0, s>>>(model_ids, n, table, p.h, p.perm);
+  if (id_kind == 1) scatter(u16); else if (id_kind == 2) scatter(u8); else scatter(i32);
   const int64_t mt = p.max[0] > p.max[1] ? p.max[0] : p.max[1];
   group_tiles<<<(unsigned)((mt + 255) / 256), 256, 0, s>>>(p.h, p.max[0], p.max[1], p.tm[0],
                                                            p.tb[0], p.tc[0], p.tm[1], p.tb[1],

@@ -76,7 +76,8 @@ cudaError_t launch_mlp_tc(const void *in, int in_kind, int prec, const TileSched
 // Grouping for infer_multi (group.cu).
 size_t group_workspace_bytes(int64_t n);
 int64_t group_max_tiles(int64_t n, int tile_rows);
-cudaError_t launch_group(int64_t n, const int32_t *model_ids, const DevModel *table,
+// id_kind: 0 int32, 1 uint16, 2 uint8 (flags bits 8..9)
+cudaError_t launch_group(int64_t n, const void *model_ids, int id_kind, const DevModel *table,
                          void *ws, int tile_rows, cudaStream_t s);
 // which = 0: 64-row FP32 tiles, 1: 256-row tensor-core tiles
 void group_sched(void *ws, int64_t n, int which, const DevModel *table, TileSched *ts);

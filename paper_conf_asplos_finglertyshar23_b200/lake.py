@@ -23,6 +23,7 @@ LAKE_ARCH_NN, LAKE_ARCH_NN1, LAKE_ARCH_NN2 = 0, 1, 2
 LAKE_IN_DIGITS, LAKE_IN_RAW = 0x00, 0x01
 LAKE_PREC_FP32, LAKE_PREC_F16, LAKE_PREC_BF16, LAKE_PREC_TF32, LAKE_PREC_AUTO = (
     0x00, 0x10, 0x20, 0x30, 0x70)
+LAKE_IDS_I32, LAKE_IDS_U16, LAKE_IDS_U8, LAKE_IDS_MASK = 0x000, 0x100, 0x200, 0x300
 LAKE_MAX_MODELS = 1024
 LAKE_SERVER_MAX_BATCH = 64
 LAKE_AUTO_TC_MIN_N = {0: 8192, 1: 1, 2: 1}  # defaults (include/lake_linnos.h)

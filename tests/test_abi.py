@@ -143,3 +143,13 @@ def test_mlp_family_host_validation():
     assert L.lake_mlp_unload(-1, 0) == lake.LAKE_ERR_INVAL
     assert L.lake_mlp_unload(5, 0) == lake.LAKE_ERR_NOMODEL
     assert L.lake_mlp_model_shape(5, 0, None, None, None) == lake.LAKE_ERR_INVAL
+
+
+def test_id_width_flags_validated_on_host():
+    """bits 8..9 select the model-id element type; 0x300 and unknown bits are rejected."""
+    L = lake.lib()
+    bad = lake.LAKE_IN_RAW | lake.LAKE_IDS_MASK
+    assert L.lake_linnos_infer_multi(16, bad, 10, 16, 16, None, 16, 1 << 20, None) == lake.LAKE_ERR_INVAL
+    assert L.lake_linnos_infer_multi(16, 0x400 | lake.LAKE_IN_RAW, 10, 16, 16, None, 16, 1 << 20,
+                                     None) == lake.LAKE_ERR_INVAL
+    assert L.lake_linnos_infer_host(16, bad, 10, 0, 16, 16, None, 16, 1 << 30, None) == lake.LAKE_ERR_INVAL

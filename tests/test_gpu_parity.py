@@ -224,6 +224,39 @@ def test_multi_unknown_ids(multi_models):
     assert np.array_equal(dec, rdec)
 
 
+def _multi_ids(raw, ids, flags):
+    """infer_multi with model ids already in the element type flags selects."""
+    import torch
+    n = raw.shape[0]
+    x = cuda(raw)
+    d_ids = torch.from_numpy(np.ascontiguousarray(ids)).to("cuda:0")
+    dec = torch.full((n,), 7, dtype=torch.uint8, device="cuda:0")
+    lg = torch.full((n, 2), 12345.0, dtype=torch.float32, device="cuda:0")
+    wsb = lake.workspace_bytes(n)
+    ws = torch.empty(max(wsb, 1), dtype=torch.uint8, device="cuda:0")
+    lake.infer_multi(x, flags, n, d_ids, dec, lg, ws, wsb)
+    unk = lake.multi_status(ws, wsb)
+    torch.cuda.synchronize()
+    return lg.cpu().numpy(), dec.cpu().numpy(), unk
+
+
+@pytest.mark.parametrize("kind", ["u8", "u16"])
+def test_multi_narrow_ids(multi_models, kind):
+    """LAKE_IDS_U8 / _U16: the same grouping and results as int32 ids, bit for bit,
+    including ids that name no loaded model."""
+    raw = _trace(20000, seed=31)
+    rng = np.random.default_rng(2)
+    pool = [100, 101, 102, 7, 255] + ([5000, 65535] if kind == "u16" else [])
+    ids = rng.choice(np.array(pool), size=raw.shape[0])
+    dt, fl = (np.uint8, lake.LAKE_IDS_U8) if kind == "u8" else (np.uint16, lake.LAKE_IDS_U16)
+    for prec in (lake.LAKE_PREC_FP32, lake.LAKE_PREC_F16):
+        lg, dec, unk = run_multi(raw, ids.astype(np.int32), lake.LAKE_IN_RAW | prec)
+        lg2, dec2, unk2 = _multi_ids(raw, ids.astype(dt), lake.LAKE_IN_RAW | prec | fl)
+        assert unk2 == unk == int((~np.isin(ids, [100, 101, 102])).sum())
+        assert np.array_equal(dec2, dec)
+        assert np.array_equal(lg2.view(np.uint32), lg.view(np.uint32))
+
+
 def test_multi_order_invariance(multi_models):
     raw, mids = inputs.multi_device_trace(9000, 3, seed_base=500, rerate=3.0)
     ids = np.array(list(multi_models))[mids]
@@ -313,11 +346,11 @@ def test_c3_full_size_sampled(prec):
 
 
 # ------------------------------------------------------------------------- host-buffer path
-def _host_call(raw, flags, model_id=-1, ids=None, logits=True):
+def _host_call(raw, flags, model_id=-1, ids=None, logits=True, id_dtype=np.int32):
     import torch
     n = raw.shape[0]
     h_in = torch.from_numpy(np.ascontiguousarray(raw).view(np.int32)).pin_memory()
-    h_ids = torch.from_numpy(ids.astype(np.int32)).pin_memory() if ids is not None else None
+    h_ids = torch.from_numpy(ids.astype(id_dtype)).pin_memory() if ids is not None else None
     h_dec = torch.full((n,), 7, dtype=torch.uint8).pin_memory()
     h_lg = torch.full((n, 2), 1234.0, dtype=torch.float32).pin_memory() if logits else None
     sb = lake.host_staging_bytes(n, flags)
@@ -342,6 +375,18 @@ def test_infer_host_pipelined_multi_equals_device(many_models):
     ids = np.array(list(many_models))[mids]
     lg, dec = _host_call(raw, lake.LAKE_IN_RAW | lake.LAKE_PREC_F16, ids=ids)
     dlg, ddec, _ = run_multi(raw, ids, lake.LAKE_IN_RAW | lake.LAKE_PREC_F16)
+    assert np.array_equal(dec, ddec)
+    assert np.array_equal(lg.view(np.uint32), dlg.view(np.uint32))
+
+
+@pytest.mark.parametrize("n", [3000, (1 << 21) + 777])
+def test_infer_host_u8_ids_equals_device(many_models, n):
+    """Host path with one-byte model ids (zero-copy size and the pipelined chunks)."""
+    raw, mids = inputs.multi_device_trace(n, 6, seed_base=2100, rerate=3.0)
+    ids = np.array(list(many_models))[mids]
+    fl = lake.LAKE_IN_RAW | lake.LAKE_PREC_F16
+    lg, dec = _host_call(raw, fl | lake.LAKE_IDS_U8, ids=ids, id_dtype=np.uint8)
+    dlg, ddec, _ = run_multi(raw, ids, fl)
     assert np.array_equal(dec, ddec)
     assert np.array_equal(lg.view(np.uint32), dlg.view(np.uint32))
 
