@@ -119,7 +119,7 @@ constexpr uint32_t kRedBytes = (kEpiPerQ - 1) * 128 * 2 * 4;  // output-layer pa
 __host__ __device__ constexpr uint32_t align1k(uint32_t x) { return (x + 1023u) & ~1023u; }
 
 struct Layout {
-  uint32_t h, x, prm, red, bar, total;
+  uint32_t h, x, prm, red, prm0, red0, bar, total;
 };
 __host__ __device__ constexpr Layout tc_layout(int nh_layout) {
   Layout L{};
@@ -127,7 +127,11 @@ __host__ __device__ constexpr Layout tc_layout(int nh_layout) {
   L.x = L.h + kHBytes;
   L.prm = L.x + 2 * kXBytes;
   L.red = L.prm + kPrmFloats * 4 + kPrm2Words * 4;
-  L.bar = L.red + kRedBytes;
+  // group 0's own copy of the output-layer parameters and partial sums: with two epilogue
+  // groups, NN tiles (a single layer) are drained by the group of their accumulator buffer
+  L.prm0 = L.red + kRedBytes;
+  L.red0 = L.prm0 + kPrmFloats * 4;
+  L.bar = L.red0 + kRedBytes;
   L.total = L.bar + 256;
   return L;
 }
@@ -425,7 +429,10 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           for (uint32_t s = 0; s < kTcK0 / 16; ++s)
             ptx::mma_f16_cg2(d, xd + s * kStep, w0desc + s * kStep, idesc, s);
           ptx::mma_commit_cg2(bar(B_XEMPTY + xb), 0x3);
-          ptx::mma_commit_cg2(bar((kEpiGroups == 2 && nh == 1 ? B_DFULLX : B_DFULL) + b), 0x3);
+          // NN: the accumulator's buffer picks the draining group (b0 -> group 0, b1 -> 1),
+          // so both groups convert logits and two NN tiles are drained at once
+          ptx::mma_commit_cg2(bar((kEpiGroups == 2 && nh == 1 && b == 1 ? B_DFULLX : B_DFULL) + b),
+                              0x3);
           LAKE_TEV(T_COMMIT, it, 0, 0);
           ++g;
         }
@@ -533,17 +540,17 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           if (IN_KIND == LAKE_IN_RAW) {
             // digit values 0..9 are exact in fp16 and bf16
             digitize_record(rec[half], [&](int k, uint32_t dg) {
-              const float v = (float)dg;
-              const uint16_t hbits = PREC == 0 ? __half_as_ushort(__float2half_rn(v))
-                                               : __bfloat16_as_ushort(__float2bfloat16_rn(v));
+              // one integer -> fp16 / bf16 conversion (I2F.F16): 0..9 are exact in both
+              const uint16_t hbits = PREC == 0 ? __half_as_ushort(__uint2half_rn(dg))
+                                               : __bfloat16_as_ushort(__uint2bfloat16_rn(dg));
               w[k >> 1] |= (uint32_t)hbits << ((k & 1) * 16);
             });
           } else {
 #pragma unroll
             for (int k = 0; k < 31; ++k) {
-              const float v = (float)((rec[half][k >> 2] >> ((k & 3) * 8)) & 0xFFu);
-              const uint16_t hbits = PREC == 0 ? __half_as_ushort(__float2half_rn(v))
-                                               : __bfloat16_as_ushort(__float2bfloat16_rn(v));
+              const uint32_t v = (rec[half][k >> 2] >> ((k & 3) * 8)) & 0xFFu;  // 0..255: exact
+              const uint16_t hbits = PREC == 0 ? __half_as_ushort(__uint2half_rn(v))
+                                               : __bfloat16_as_ushort(__uint2bfloat16_rn(v));
               w[k >> 1] |= (uint32_t)hbits << ((k & 1) * 16);
             }
           }
@@ -573,9 +580,11 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
     const uint32_t hready_leader0 = ptx::mapa(bar(B_HREADY), 0);
     const uint32_t tempty_leader0 = ptx::mapa(bar(B_TEMPTY), 0);
     const uint32_t hrow = sbase + L.h + row * 16;
-    float *prm = reinterpret_cast<float *>(smem + L.prm);    // last bias | W_out | b_out
+    const bool own0 = kEpiGroups == 2 && gy == 0;  // group 0's private output-layer copy
+    float *prm = reinterpret_cast<float *>(smem + (own0 ? L.prm0 : L.prm));  // last b | W_out | b_out
     uint32_t *prm2 = reinterpret_cast<uint32_t *>(smem + L.prm + kPrmFloats * 4);
-    float *red = reinterpret_cast<float *>(smem + L.red);
+    float *red = reinterpret_cast<float *>(smem + (own0 ? L.red0 : L.red));
+    const uint32_t red_bar = (own0 ? 8 : 4) + q;  // named barrier of this quadrant's reduction
     const DevModel *cur = nullptr;
     uint32_t g = 0, d_phase = 0, dx_phase = 0;  // phase bits per accumulator buffer
     int64_t it = 0;
@@ -599,7 +608,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
             prm2[i] = PREC == 0 ? ptx::pack_f16(bf.x, bf.y) : ptx::pack_bf16(bf.x, bf.y);
           }
         }
-        if (do_last) {
+        if (do_last || (kEpiGroups == 2 && nh == 1)) {
           const float4 *src = reinterpret_cast<const float4 *>(ti.model->b[nh - 1]);
           for (uint32_t i = et; i < kPrmFloats / 4; i += NG)
             reinterpret_cast<float4 *>(prm)[i] = __ldg(src + i);
@@ -610,9 +619,10 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       const float *wo = prm + kHidden;
       for (int l = 0; l < nh; ++l, ++g) {
         const bool last = (l + 1 == nh);
-        if (!(last ? do_last : do_h)) continue;
         const uint32_t b = g & 1;
-        if (kEpiGroups == 2 && last) {
+        const bool nn2 = kEpiGroups == 2 && nh == 1;  // NN: buffer b is drained by group b
+        if (nn2 ? gy != b : !(last ? do_last : do_h)) continue;
+        if (kEpiGroups == 2 && (nn2 ? b == 1 : last)) {
           ptx::mbar_wait(bar(B_DFULLX + b), (dx_phase >> b) & 1);
           dx_phase ^= (1u << b);
         } else {
@@ -708,7 +718,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
             rd[0] = p0;
             rd[1] = p1;
           }
-          ptx::named_bar_sync(4 + q, 32 * kEpiPerQ);
+          ptx::named_bar_sync(red_bar, 32 * kEpiPerQ);
           if (hh == 0) {
 #pragma unroll
             for (uint32_t j = 0; j + 1 < kEpiPerQ; ++j) {
@@ -718,7 +728,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           }
           // close the exchange before the partial sums are overwritten by the next tile
           // (single group: only NN lacks a later ordering point)
-          if (kEpiGroups == 2 || nh == 1) ptx::named_bar_sync(4 + q, 32 * kEpiPerQ);
+          if (kEpiGroups == 2 || nh == 1) ptx::named_bar_sync(red_bar, 32 * kEpiPerQ);
           if (hh == 0) {
             const float l0 = p0 + wo[2 * kHidden + 0];
             const float l1 = p1 + wo[2 * kHidden + 1];

@@ -21,7 +21,7 @@ CAP = 1 << 16
 cfg = sys.argv[1] if len(sys.argv) > 1 else "C5"
 prec = sys.argv[2] if len(sys.argv) > 2 else "f16"
 torch.cuda.set_device(0)
-w = inputs.workload(cfg)
+w = inputs.workload(cfg, arch=int(sys.argv[3]) if len(sys.argv) > 3 else None)
 for m, (a, blob) in w["models"].items():
     lake.load_weights(m, a, blob, 0)
 n = w["raw"].shape[0]
