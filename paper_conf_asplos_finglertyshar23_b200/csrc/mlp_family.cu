@@ -29,6 +29,7 @@
 
 #include "../../include/lake_mlp.h"
 #include "lake_internal.h"
+#include "lake_ptx.cuh"
 
 namespace lake {
 namespace {
@@ -288,35 +289,51 @@ mlp_family_kernel(const float *__restrict__ x, int64_t n, const __grid_constant_
     fam_smem4[i] = __ldg(reinterpret_cast<const float4 *>(img) + i);
 
   const int64_t n_tiles = (n + ROWS - 1) / ROWS;
-  // asynchronous copy of one tile's rows (contiguous cnt*W0 floats) into a staging buffer;
-  // tile * ROWS * W0 * 4 bytes is a multiple of 16, so 16-byte copies line up when x does
-  auto stage = [&](int64_t tile, float *dst) {
+  // One tile's rows are cnt*W0 contiguous floats, and tile * ROWS * W0 * 4 bytes is a
+  // multiple of 16: with a 16-byte aligned x, one thread moves the tile with a single bulk
+  // copy (TMA engine, completion on an mbarrier) plus at most 3 tail floats; otherwise every
+  // thread issues 4-byte cp.async copies.
+  __shared__ __align__(8) uint64_t fam_bar[2];
+  const uint32_t bar0 = ptx::smem_u32(&fam_bar[0]);
+  if (vec && tid == 0) {
+    ptx::mbar_init(bar0, 1);
+    ptx::mbar_init(bar0 + 8, 1);
+    ptx::fence_mbar_init();
+  }
+  auto stage = [&](int64_t tile, float *dst, uint32_t bar) {
     const int64_t row0 = tile * ROWS;
     const int cnt = (int)((n - row0) < ROWS ? (n - row0) : ROWS);
     const int nf = cnt * W0;
     const float *src = x + row0 * W0;
-    int done = 0;
     if (vec) {
-      const int n4 = nf >> 2;
-      for (int i = tid; i < n4; i += kFamThreads)
-        __pipeline_memcpy_async(dst + 4 * i, src + 4 * i, 16);
-      done = n4 << 2;
+      if (tid == 0) {
+        const uint32_t bulk = (uint32_t)(nf & ~3) * 4;
+        ptx::mbar_arrive_expect_tx(bar, bulk);
+        if (bulk) ptx::bulk_g2s(ptx::smem_u32(dst), src, bulk, bar);
+      }
+      const int i = (nf & ~3) + tid;  // tail: plain loads, made visible by __syncthreads
+      if (i < nf) dst[i] = __ldg(src + i);
+    } else {
+      for (int i = tid; i < nf; i += kFamThreads)
+        __pipeline_memcpy_async(dst + i, src + i, 4);
+      __pipeline_commit();
     }
-    for (int i = done + tid; i < nf; i += kFamThreads)
-      __pipeline_memcpy_async(dst + i, src + i, 4);
-    __pipeline_commit();
   };
-  if ((int64_t)blockIdx.x < n_tiles) stage(blockIdx.x, sxb0);
+  __syncthreads();  // barrier init visible before the first copy
+  if ((int64_t)blockIdx.x < n_tiles) stage(blockIdx.x, sxb0, bar0);
 
   int it = 0;
   for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x, ++it) {
     const int64_t row0 = tile * ROWS;
     const int cnt = (int)((n - row0) < ROWS ? (n - row0) : ROWS);
     __syncthreads();  // image copied; every thread is done with the previous tile's rows
-    if (tile + gridDim.x < n_tiles) stage(tile + gridDim.x, (it & 1) ? sxb0 : sxb1);
-    else __pipeline_commit();
-    __pipeline_wait_prior(1);  // this thread's copies of the current tile have landed
-    __syncthreads();           // ... and everyone's
+    if (tile + gridDim.x < n_tiles)
+      stage(tile + gridDim.x, (it & 1) ? sxb0 : sxb1, bar0 + ((it + 1) & 1) * 8);
+    else if (!vec)
+      __pipeline_commit();
+    if (vec) ptx::mbar_wait(bar0 + (it & 1) * 8, (uint32_t)((it >> 1) & 1));
+    else __pipeline_wait_prior(1);  // this thread's copies of the current tile have landed
+    __syncthreads();                // ... and everyone's
     const float *sx = (it & 1) ? sxb1 : sxb0;
     int sxs = W0;
     if (!(W0 & 1)) {  // even width: re-lay rows at an odd stride (bank-conflict-free reads)
@@ -391,7 +408,7 @@ cudaError_t fam_launch(const float *x, int64_t n, const FamModel &m, int32_t *cl
   dev &= kFamMaxDevices - 1;
   if (!attr_set[dev]) {
     cudaError_t e = cudaFuncSetAttribute(mlp_family_kernel<Body, RPT>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, 226 * 1024);  // + static barriers
     if (e != cudaSuccess) return e;
     attr_set[dev] = true;
   }

@@ -14,4 +14,8 @@ timeout 600 ncu --set full --clock-control none --import-source on -k regex:mlp_
     > gpurun_out/full_fp32_$TAG.out 2>&1
 timeout 300 ncu --set full --clock-control none -k regex:digitize_kernel -c 1 \
     -o gpurun_out/full_dig_$TAG python scripts/run_digitize.py > gpurun_out/full_dig_$TAG.out 2>&1
+for m in mllb kml; do
+  timeout 300 ncu --set full --clock-control none --import-source on -k regex:mlp_family -s 1 -c 1 \
+      -o gpurun_out/full_fam${m}_$TAG python scripts/run_family.py $m > gpurun_out/full_fam${m}_$TAG.out 2>&1
+done
 echo done

@@ -158,3 +158,25 @@ def test_full_size_sampled(name, kernel_path):
     ro, rc = oracle.mlp_family(widths, act, blob, x[rows], nthreads=0)
     _check(act, o[rows], c[rows], ro, rc)
     lake.mlp_unload(4, 0)
+
+
+@pytest.mark.parametrize("name", ["mllb", "kml"])
+def test_unaligned_input_rows(name, kernel_path):
+    """x not 16-byte aligned: the kernel falls back from the bulk (TMA) row copy to 4-byte
+    cp.async copies; results are the same."""
+    widths, act = SHAPES[name]
+    blob = family.weights(widths, 6)
+    lake.mlp_load(5, widths, act, blob, 0)
+    n = 50000 + 3
+    x = family.features(n, widths[0], 77)
+    buf = torch.zeros(n * widths[0] + 1, dtype=torch.float32, device=DEV)
+    buf[1:] = torch.from_numpy(x.ravel()).to(DEV)
+    xd = buf[1:]
+    assert xd.data_ptr() % 16 != 0
+    cls = torch.full((n,), -7, dtype=torch.int32, device=DEV)
+    out = torch.full((n, widths[-1]), 12345.0, dtype=torch.float32, device=DEV)
+    lake.mlp_infer(xd, n, 5, cls, out)
+    torch.cuda.synchronize()
+    ro, rc = oracle.mlp_family(widths, act, blob, x, nthreads=0)
+    _check(act, out.cpu().numpy(), cls.cpu().numpy(), ro, rc)
+    lake.mlp_unload(5, 0)
