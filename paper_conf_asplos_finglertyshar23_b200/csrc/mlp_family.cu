@@ -35,6 +35,14 @@ namespace lake {
 namespace {
 
 constexpr int kFamThreads = 128;
+// rows per thread of the compile-time-shape kernels for large batches (each weight LDS.128
+// then feeds 4 * RPT FMAs); A/B on B200: MLLB 2 -> 4 rows +12%
+#ifndef LAKE_FAM_RPT
+#define LAKE_FAM_RPT 4
+#endif
+#ifndef LAKE_FAM_RPT_KML
+#define LAKE_FAM_RPT_KML 2
+#endif
 constexpr int kFamMaxDevices = 64;
 
 struct FamModel {
@@ -613,10 +621,10 @@ int lake_mlp_infer(const float *x, int64_t n, int32_t model_id, int32_t *classes
     generic = g_fam_force_generic;
   }
   if (m.fixed == 1 && !generic)
-    e = big ? fam_launch<FixedBody<MllbShape>, 2>(x, n, m, classes, out, s, sms)
+    e = big ? fam_launch<FixedBody<MllbShape>, LAKE_FAM_RPT>(x, n, m, classes, out, s, sms)
             : fam_launch<FixedBody<MllbShape>, 1>(x, n, m, classes, out, s, sms);
   else if (m.fixed == 2 && !generic)
-    e = big ? fam_launch<FixedBody<KmlShape>, 2>(x, n, m, classes, out, s, sms)
+    e = big ? fam_launch<FixedBody<KmlShape>, LAKE_FAM_RPT_KML>(x, n, m, classes, out, s, sms)
             : fam_launch<FixedBody<KmlShape>, 1>(x, n, m, classes, out, s, sms);
   else if (maxw == 16)
     e = big ? fam_launch<GenericBody<16>, 2>(x, n, m, classes, out, s, sms)
