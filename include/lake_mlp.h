@@ -46,7 +46,9 @@ extern "C" {
 /* Hidden-layer activation; the output layer is always the identity. */
 enum lake_mlp_act {
     LAKE_ACT_RELU = 0,    /* h = (z > 0.0f) ? z : +0.0f                          (R15) */
-    LAKE_ACT_SIGMOID = 1  /* h = 1.0f / (1.0f + expf(-z)), IEEE division, full expf (R27) */
+    LAKE_ACT_SIGMOID = 1  /* h = 1 / (1 + exp(-z)); computed on the SFU (ex2.approx,
+                             rcp.approx): outputs within 1e-5 relative of the binary32
+                             definition 1.0f / (1.0f + expf(-z)) (R27)                 */
 };
 
 /* Exact blob length in floats for a shape, or 0 if the shape is invalid:

@@ -1,8 +1,8 @@
 """GPU parity of the NEXT-4 MLP family (include/lake_mlp.h) against oracle.mlp_family.
 
 ReLU models: outputs and classes bit-exact (same operation order, R15).
-Sigmoid models: the kernel's expf / IEEE division and glibc's expf differ by a few ulp,
-so outputs are compared within 1e-5 relative (S19 form: |d| / max(|ref|, rms(ref))) and
+Sigmoid models: the kernel computes sigmoid on the SFU (ex2.approx / rcp.approx), the oracle
+with glibc expf and IEEE division, so outputs are compared within 1e-5 relative (S19 form: |d| / max(|ref|, rms(ref))) and
 classes must agree wherever the oracle's top-two margin exceeds 1e-4 (R27/R28).
 Inputs come from the seeded generators; expected values only from oracle/."""
 import numpy as np
