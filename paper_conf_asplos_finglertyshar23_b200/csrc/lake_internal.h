@@ -18,7 +18,10 @@ constexpr int kMaxHiddenLayers = 3;
 // groups: position p(j) = (jj/4)*128 + tc*4 + (jj%4) with tc = j%32, jj = j/32.
 constexpr int kF32TileM = 64;       // I/Os per CTA tile
 constexpr int kF32Threads = 256;
-constexpr int kF32KChunk = 16;      // rows of W^T staged per pipeline stage
+#ifndef LAKE_F32_KC
+#define LAKE_F32_KC 64
+#endif
+constexpr int kF32KChunk = LAKE_F32_KC;  // rows of W^T staged per pipeline stage
 constexpr int kF32ActStride = 68;   // floats per activation row in SMEM (64 + 4 pad)
 
 // ---- tcgen05 path (mlp_tc.cu) ------------------------------------------------------------

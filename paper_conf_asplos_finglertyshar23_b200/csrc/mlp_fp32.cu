@@ -13,7 +13,8 @@
 // Each accumulator is summed over k strictly in order (that is what a K-loop GEMM does),
 // so the tiling changes nothing numerically. Activations live transposed in SMEM
 // (act[k][row], row stride 68 floats: broadcast A reads, conflict-free epilogue stores);
-// weights stream through a 2-stage cp.async pipeline in 16-row chunks of W^T whose columns
+// weights stream through a 2-stage cp.async pipeline in 64-row chunks of W^T (16 for the
+// 16-row latency tile), activations are updated in place, and W^T columns
 // were permuted at load time so each thread's 8 columns are two float4s.
 // The 2-wide output layer is one sequential fmaf chain per (row, class).
 #include <cuda_pipeline.h>
@@ -24,7 +25,14 @@
 namespace lake {
 namespace {
 
-constexpr int KC = kF32KChunk;
+#ifndef LAKE_F32_UNROLL
+#define LAKE_F32_UNROLL 4
+#endif
+constexpr int kF32Unroll = LAKE_F32_UNROLL;  // k-loop unroll of the RM = 8 tile
+#ifndef LAKE_F32_ACT_BUFS
+#define LAKE_F32_ACT_BUFS 1
+#endif
+constexpr int kF32ActBufs = LAKE_F32_ACT_BUFS;  // 1: in place (frees SMEM for KC = 64)
 
 template <int RM>
 struct F32Cfg {
@@ -33,12 +41,17 @@ struct F32Cfg {
   // activation row stride: float4-aligned with a 4-float pad for RM = 8 (conflict-free
   // float4 epilogue stores), odd for RM = 2 (conflict-free scalar stores)
   static constexpr int S = RM == 8 ? kF32ActStride : M + 1;
+  // rows of W^T per pipeline stage: 64 for the throughput tile (4 syncs per 256-wide layer;
+  // A/B on B200: 16 -> 64 rows +6% on NN+2), 16 for the 16-row latency tile
+  static constexpr int KC = RM == 8 ? kF32KChunk : 16;
 };
 
 template <int RM>
 struct F32Smem {
-  float act[2][kHidden][F32Cfg<RM>::S];  // transposed activations, ping-pong
-  float w[2][KC][kHidden];               // W^T chunk staging (permuted columns)
+  // transposed activations, updated in place: a layer's outputs are written only after
+  // the __syncthreads that closes its last K chunk, i.e. once every input has been read
+  float act[kF32ActBufs][kHidden][F32Cfg<RM>::S];
+  float w[2][F32Cfg<RM>::KC][kHidden];   // W^T chunk staging (permuted columns)
   float wout[2][kHidden];
   float bout[4];
   int32_t rows[F32Cfg<RM>::M];           // I/O index per tile row, -1 = padding
@@ -59,7 +72,7 @@ __global__ void __launch_bounds__(kF32Threads, 1)
 mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
                 uint8_t *__restrict__ decisions,
                 float *__restrict__ logits) {
-  constexpr int M = F32Cfg<RM>::M, S = F32Cfg<RM>::S, HR = F32Cfg<RM>::HR;
+  constexpr int M = F32Cfg<RM>::M, S = F32Cfg<RM>::S, HR = F32Cfg<RM>::HR, KC = F32Cfg<RM>::KC;
   extern __shared__ __align__(16) uint8_t smem_raw[];
   F32Smem<RM> &sm = *reinterpret_cast<F32Smem<RM> *>(smem_raw);
   const int tid = threadIdx.x;
@@ -119,18 +132,19 @@ mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched t
       const int K = (l == 0) ? kInputs : kHidden;         // strict: layer 0 sums 31 terms
       const int Kst = (l == 0) ? 32 : kHidden;            // staged rows (row 31 is zero)
       const float *wt = mp->wt[l];
-      const float (*ain)[S] = sm.act[l & 1];
-      float (*aout)[S] = sm.act[(l + 1) & 1];
+      const float (*ain)[S] = sm.act[kF32ActBufs == 2 ? (l & 1) : 0];
+      float (*aout)[S] = sm.act[kF32ActBufs == 2 ? ((l + 1) & 1) : 0];
       float acc[RM][8];
 #pragma unroll
       for (int i = 0; i < RM; ++i)
 #pragma unroll
         for (int j = 0; j < 8; ++j) acc[i][j] = 0.0f;
-      const int nch = Kst / KC;
-      stage_chunk(sm.w[0], wt, KC);
+      const int nch = (Kst + KC - 1) / KC;  // layer 0 stages its 32 rows even when KC > 32
+      stage_chunk(sm.w[0], wt, Kst < KC ? Kst : KC);
       for (int c = 0; c < nch; ++c) {
         if (c + 1 < nch) {
-          stage_chunk(sm.w[(c + 1) & 1], wt + (int64_t)(c + 1) * KC * kHidden, KC);
+          const int rows = (Kst - (c + 1) * KC) < KC ? (Kst - (c + 1) * KC) : KC;
+          stage_chunk(sm.w[(c + 1) & 1], wt + (int64_t)(c + 1) * KC * kHidden, rows);
           __pipeline_wait_prior(1);
         } else {
           __pipeline_wait_prior(0);
@@ -138,7 +152,7 @@ mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched t
         __syncthreads();
         const float (*wc)[kHidden] = sm.w[c & 1];
         const int kmax = (K - c * KC) < KC ? (K - c * KC) : KC;
-#pragma unroll 4
+#pragma unroll kF32Unroll
         for (int kk = 0; kk < kmax; ++kk) {
           const int k = c * KC + kk;
           float av[RM];
@@ -193,7 +207,7 @@ mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched t
     // ---- output layer (2 neurons, identity) + decision ------------------------------------
     if (tid < 2 * M) {
       const int r = tid >> 1, c = tid & 1;
-      const float (*h)[S] = sm.act[nh & 1];
+      const float (*h)[S] = sm.act[kF32ActBufs == 2 ? (nh & 1) : 0];
       float acc = 0.0f;
 #pragma unroll 8
       for (int k = 0; k < kHidden; ++k) acc = __fmaf_rn(h[k][r], sm.wout[c][k], acc);
