@@ -345,6 +345,40 @@ def test_c3_full_size_sampled(prec):
         assert met["agreement"] >= 0.999, met
 
 
+@pytest.mark.parametrize("prec", [lake.LAKE_PREC_F16, lake.LAKE_PREC_FP32])
+def test_c5_full_size_sampled(prec):
+    """The bench's own configuration (C5: 64 per-SSD NN+2 models, 2^24 interleaved I/Os,
+    lake_linnos_infer_multi = grouping + fused kernel), checked on sampled I/Os that the
+    oracle scores one by one with each I/O's own model."""
+    w = inputs.workload("C5")
+    raw, ids = w["raw"], w["model_ids"]
+    n = raw.shape[0]
+    assert n == 1 << 24 and len(w["models"]) == 64
+    for m, (a, blob) in w["models"].items():
+        lake.load_weights(300 + m, a, blob, 0)
+    try:
+        lg, dec, unk = run_multi(raw, (ids + 300).astype(np.int32), lake.LAKE_IN_RAW | prec)
+    finally:
+        for m in w["models"]:
+            lake.unload(300 + m, 0)
+    assert unk == 0
+    rng = np.random.default_rng(5)
+    smp = np.unique(np.concatenate([rng.choice(n, 6000, replace=False), np.arange(n - 200, n)]))
+    rlg = np.zeros((smp.size, 2), np.float32)
+    rdec = np.zeros(smp.size, np.uint8)
+    for m, (a, blob) in w["models"].items():
+        sel = np.nonzero(ids[smp] == m)[0]
+        if sel.size:
+            rlg[sel], rdec[sel] = oracle.infer_raw(a, blob, raw[smp[sel]], nthreads=0)
+    if prec == lake.LAKE_PREC_FP32:
+        assert np.array_equal(dec[smp], rdec)
+        assert np.array_equal(lg[smp].view(np.uint32), rlg.view(np.uint32))
+    else:
+        met = tc_metrics(lg[smp], dec[smp], rlg, rdec)
+        assert met["max_rel"] <= 2e-2 and met["max_disagree_margin"] < 5e-2, met
+        assert met["agreement"] >= 0.999, met
+
+
 # ------------------------------------------------------------------------- host-buffer path
 def _host_call(raw, flags, model_id=-1, ids=None, logits=True, id_dtype=np.int32):
     import torch
