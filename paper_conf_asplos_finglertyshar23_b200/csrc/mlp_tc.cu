@@ -401,8 +401,28 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       };
       TileInfo nxt;
       if (t_begin < t_end) nxt = tile_info<PREC>(ts, t_begin);
+#ifndef LAKE_NO_MMA_SCHED2
+#define LAKE_MMA_SCHED2 1
+#endif
+#ifdef LAKE_MMA_SCHED2
+      // schedule entries two tiles ahead: the model slot of tile t+2 is loaded at the top of
+      // tile t and the dependent model-table loads of tile t+1 are issued there too, from a
+      // slot loaded one tile earlier, so no load result is waited for on the tile boundary
+      auto slot_of = [&](int64_t tt) -> int32_t { return ts.tile_model ? ts.tile_model[tt] : -1; };
+      int32_t slot_n = (t_begin + 1 < t_end) ? slot_of(t_begin + 1) : -1;
+#endif
       for (int64_t t = t_begin; t < t_end; ++t, ++it) {
-#ifdef LAKE_NO_PREFETCH
+#ifdef LAKE_MMA_SCHED2
+        const TileInfo ti = nxt;
+        const int32_t slot_nn = (t + 2 < t_end) ? slot_of(t + 2) : -1;
+        if (t + 1 < t_end) {
+          const DevModel *mm = slot_n >= 0 ? &ts.table[slot_n] : &ts.model;
+          nxt.model = mm;
+          nxt.img = mm->tc_img[PREC];
+          nxt.nh = mm->nh;
+        }
+        slot_n = slot_nn;
+#elif defined(LAKE_NO_PREFETCH)
         const TileInfo ti = tile_info<PREC>(ts, t);
         if (t + 1 < t_end) nxt = tile_info<PREC>(ts, t + 1);
 #else
