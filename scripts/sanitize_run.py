@@ -41,6 +41,24 @@ h_dec = torch.empty(3000, dtype=torch.uint8).pin_memory()
 sb = lake.host_staging_bytes(3000, lake.LAKE_IN_RAW)
 stg = torch.empty(sb, dtype=torch.uint8, device=dev)
 lake.infer_host(h_in, lake.LAKE_IN_RAW | lake.LAKE_PREC_F16, 3000, 3, None, h_dec, None, stg, sb)
+# one-byte model ids through the host path; NEXT-4 MLP family (fixed-shape and generic
+# kernels, aligned bulk-copy staging and unaligned cp.async staging, ragged tiles)
+h_ids8 = torch.from_numpy(np.random.default_rng(1).integers(1, 4, 3000).astype(np.uint8)).pin_memory()
+lake.infer_host(h_in, lake.LAKE_IN_RAW | lake.LAKE_PREC_F16 | lake.LAKE_IDS_U8, 3000, -1, h_ids8,
+                h_dec, None, stg, sb)
+from paper_conf_asplos_finglertyshar23_b200.inputs import family  # noqa: E402
+for mid, (shape, act) in enumerate((((15, 10, 10, 2), 0), ((5, 15, 15, 4), 1), ((16, 8, 5), 0))):
+    lake.mlp_load(mid, shape, act, family.weights(shape, mid), 0)
+    fx = torch.from_numpy(family.features(40001, shape[0], mid)).to(dev)
+    cls = torch.empty(40001, dtype=torch.int32, device=dev)
+    fo = torch.empty((40001, shape[-1]), dtype=torch.float32, device=dev)
+    for n in (1, 129, 40001):
+        lake.mlp_infer(fx, n, mid, cls, fo)
+    flat = fx.flatten()
+    lake.mlp_infer(flat[1:1 + 999 * shape[0]], 999, mid, cls, fo)  # 4-byte aligned only
+    prev = lake.mlp_force_generic(True)
+    lake.mlp_infer(fx, 40001, mid, cls, None)
+    lake.mlp_force_generic(prev)
 torch.cuda.synchronize()
 if os.environ.get("SANITIZE_SERVER", "1") == "1":
     with lake.Server(3) as srv:
