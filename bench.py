@@ -696,9 +696,9 @@ FP32_PEAK_TFLOPS = 74.4  # 148 SM x 128 FP32 lanes x 2 FLOP x 1.965 GHz (DESIGN.
 def run_family(args):
     """NEXT-4: the MLLB / KML-shaped MLPs (include/lake_mlp.h, readings
     R25-R28). Per model: batch latency vs batch size 1..1024 (Fig. 10 / Fig. 11's range,
-    P:1436-1535): end to end through the public call with host buffers (pinned H2D of the
-    features, lake_mlp_infer, D2H of the classes, sync; host clock) and device-only (CUDA
-    events), beside the 1-thread oracle for the same batch, with the crossover batch; then
+    P:1436-1535): end to end through the public call with pinned host buffers
+    (lake_mlp_infer_host: the kernel reads the features from and writes the classes to host
+    memory, then a stream sync) and device-only (CUDA events), beside the 1-thread oracle for the same batch, with the crossover batch; then
     throughput at 2^24 rows (inputs resident in HBM, larger than L2) against the FP32 and
     HBM rooflines, and the oracle on all host cores on a bounded sample."""
     import torch
@@ -724,15 +724,12 @@ def run_family(args):
             x = np.ascontiguousarray(x_all[:b])
             h_x = torch.from_numpy(x).pin_memory()
             h_c = torch.empty(b, dtype=torch.int32).pin_memory()
-            d_x = torch.empty_like(h_x, device=dev)
+            d_x = h_x.to(dev)
             d_c = torch.empty(b, dtype=torch.int32, device=dev)
             reps, warm = 200, 20
 
-            def once():
-                d_x.copy_(h_x, non_blocking=True)
-                lake.mlp_infer(d_x, b, mid, d_c, None, stream)
-                h_c.copy_(d_c, non_blocking=True)
-                stream.synchronize()
+            def once():  # the public host-buffer call (zero-copy for pinned buffers)
+                lake.mlp_infer_host(h_x, b, mid, h_c, None, None, 0, stream)
             for _ in range(warm):
                 once()
             ts = []

@@ -84,6 +84,20 @@ int lake_mlp_unload(int32_t model_id, int32_t device);
 int lake_mlp_infer(const float *x, int64_t n, int32_t model_id, int32_t *classes, float *out,
                    void *stream);
 
+/* Device staging bytes lake_mlp_infer_host needs for n rows of width_in inputs and
+ * `classes` outputs (0 for n < 0 or a width outside 1..LAKE_MLP_MAX_WIDTH). */
+size_t lake_mlp_host_staging_bytes(int64_t n, int32_t width_in, int32_t classes);
+
+/* score_features with HOST buffers, synchronous (returns after the results are in host
+ * memory): the batch-latency path of Fig. 10 / Fig. 11 ("including data copying"). When
+ * every host buffer is pinned and mapped (UVA), the kernel reads the features from and
+ * writes the classes / outputs to host memory directly (no copy-engine round trips);
+ * otherwise it copies through d_staging (device, >= lake_mlp_host_staging_bytes).
+ *   h_x : host float[n][widths[0]]; h_classes : host int32[n]; h_out : host float[n][C]
+ *   or NULL. Errors as lake_mlp_infer, plus LAKE_ERR_NOMEM if staging is needed and short. */
+int lake_mlp_infer_host(const float *h_x, int64_t n, int32_t model_id, int32_t *h_classes,
+                        float *h_out, void *d_staging, size_t staging_bytes, void *stream);
+
 /* Shape of a loaded model: *n_layers_out and widths_out[0..n_layers] (caller provides
  * LAKE_MLP_MAX_LAYERS + 1 entries), *act_out. LAKE_ERR_NOMODEL if not loaded. */
 int lake_mlp_model_shape(int32_t model_id, int32_t device, int32_t *n_layers_out,

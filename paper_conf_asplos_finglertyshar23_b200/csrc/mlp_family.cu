@@ -578,6 +578,67 @@ int lake_mlp_unload(int32_t model_id, int32_t device) {
   return LAKE_OK;
 }
 
+size_t lake_mlp_host_staging_bytes(int64_t n, int32_t width_in, int32_t classes) {
+  if (n < 0 || width_in < 1 || width_in > LAKE_MLP_MAX_WIDTH || classes < 2 ||
+      classes > LAKE_MLP_MAX_WIDTH)
+    return 0;
+  const size_t r = (size_t)(n > 0 ? n : 1);
+  auto a256 = [](size_t x) { return (x + 255) & ~(size_t)255; };
+  return a256(r * width_in * 4) + a256(r * 4) + a256(r * classes * 4);
+}
+
+int lake_mlp_infer_host(const float *h_x, int64_t n, int32_t model_id, int32_t *h_classes,
+                        float *h_out, void *d_staging, size_t staging_bytes, void *stream) {
+  if (n < 0 || n > (int64_t)INT32_MAX) return LAKE_ERR_INVAL;
+  if (n == 0) return LAKE_OK;
+  if (!h_x || !h_classes) return LAKE_ERR_INVAL;
+  if (model_id < 0 || model_id >= LAKE_MLP_MAX_MODELS) return LAKE_ERR_NOMODEL;
+  int device = 0;
+  if (cudaGetDevice(&device) != cudaSuccess) return LAKE_ERR_CUDA;
+  if (device < 0 || device >= kFamMaxDevices) return LAKE_ERR_NOMODEL;
+  int32_t w0, C;
+  {
+    std::lock_guard<std::mutex> lk(g_fam_mu);
+    if (!g_fam[device] || !g_fam[device]->slot[model_id].loaded) return LAKE_ERR_NOMODEL;
+    const FamModel &m = g_fam[device]->slot[model_id].m;
+    w0 = m.widths[0];
+    C = m.widths[m.n_layers];
+  }
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  // zero-copy when every host buffer is pinned and mapped
+  auto mapped = [](const void *h) -> void * {
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, h) != cudaSuccess) {
+      cudaGetLastError();
+      return nullptr;
+    }
+    return (a.type == cudaMemoryTypeHost) ? a.devicePointer : nullptr;
+  };
+  void *dx = mapped(h_x), *dc = mapped(h_classes), *dout = h_out ? mapped(h_out) : nullptr;
+  int rc;
+  if (dx && dc && (!h_out || dout)) {
+    rc = lake_mlp_infer(static_cast<const float *>(dx), n, model_id, static_cast<int32_t *>(dc),
+                        static_cast<float *>(dout), stream);
+    if (rc != LAKE_OK) return rc;
+    return fam_cuda_status(cudaStreamSynchronize(s));
+  }
+  if (!d_staging || staging_bytes < lake_mlp_host_staging_bytes(n, w0, C)) return LAKE_ERR_NOMEM;
+  auto a256 = [](size_t x) { return (x + 255) & ~(size_t)255; };
+  uint8_t *b = static_cast<uint8_t *>(d_staging);
+  float *sx = reinterpret_cast<float *>(b);
+  int32_t *sc = reinterpret_cast<int32_t *>(b + a256((size_t)n * w0 * 4));
+  float *so = reinterpret_cast<float *>(b + a256((size_t)n * w0 * 4) + a256((size_t)n * 4));
+  cudaError_t e = cudaMemcpyAsync(sx, h_x, (size_t)n * w0 * 4, cudaMemcpyHostToDevice, s);
+  if (e != cudaSuccess) return fam_cuda_status(e);
+  rc = lake_mlp_infer(sx, n, model_id, sc, h_out ? so : nullptr, stream);
+  if (rc != LAKE_OK) return rc;
+  e = cudaMemcpyAsync(h_classes, sc, (size_t)n * 4, cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess && h_out)
+    e = cudaMemcpyAsync(h_out, so, (size_t)n * C * 4, cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  return fam_cuda_status(e);
+}
+
 int lake_mlp_force_generic(int32_t enable) {
   std::lock_guard<std::mutex> lk(g_fam_mu);
   const int prev = g_fam_force_generic ? 1 : 0;

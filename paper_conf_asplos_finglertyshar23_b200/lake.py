@@ -46,7 +46,8 @@ EXPORTS = (
 # every symbol include/lake_mlp.h declares (NEXT-4 MLP family)
 MLP_EXPORTS = (
     "lake_mlp_blob_floats", "lake_mlp_load", "lake_mlp_unload", "lake_mlp_infer",
-    "lake_mlp_model_shape", "lake_mlp_force_generic",
+    "lake_mlp_model_shape", "lake_mlp_force_generic", "lake_mlp_host_staging_bytes",
+    "lake_mlp_infer_host",
 )
 LAKE_ACT_RELU, LAKE_ACT_SIGMOID = 0, 1
 LAKE_MLP_MAX_LAYERS, LAKE_MLP_MAX_WIDTH, LAKE_MLP_MAX_MODELS = 4, 64, 256
@@ -102,6 +103,8 @@ def lib():
             "lake_mlp_infer": (ctypes.c_int, [P, I64, I32, P, P, P]),
             "lake_mlp_model_shape": (ctypes.c_int, [I32, I32, P, P, P]),
             "lake_mlp_force_generic": (ctypes.c_int, [I32]),
+            "lake_mlp_host_staging_bytes": (SZ, [I64, I32, I32]),
+            "lake_mlp_infer_host": (ctypes.c_int, [P, I64, I32, P, P, P, SZ, P]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -308,3 +311,14 @@ def mlp_model_shape(model_id: int, device: int):
 def mlp_force_generic(enable: bool) -> bool:
     """Route every MLP-family model through the generic kernel; returns the previous value."""
     return bool(lib().lake_mlp_force_generic(1 if enable else 0))
+
+
+def mlp_host_staging_bytes(n: int, width_in: int, classes: int) -> int:
+    return int(lib().lake_mlp_host_staging_bytes(n, width_in, classes))
+
+
+def mlp_infer_host(h_x, n: int, model_id: int, h_classes, h_out=None, d_staging=None,
+                   staging_bytes: int = 0, stream=None) -> None:
+    _check(lib().lake_mlp_infer_host(_ptr(h_x), n, model_id, _ptr(h_classes), _ptr(h_out),
+                                     _ptr(d_staging), staging_bytes, _stream(stream)),
+           "mlp_infer_host")

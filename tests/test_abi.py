@@ -143,6 +143,11 @@ def test_mlp_family_host_validation():
     assert L.lake_mlp_unload(-1, 0) == lake.LAKE_ERR_INVAL
     assert L.lake_mlp_unload(5, 0) == lake.LAKE_ERR_NOMODEL
     assert L.lake_mlp_model_shape(5, 0, None, None, None) == lake.LAKE_ERR_INVAL
+    assert lake.mlp_host_staging_bytes(1000, 15, 2) >= 1000 * (15 + 1 + 2) * 4
+    assert lake.mlp_host_staging_bytes(-1, 15, 2) == 0 and lake.mlp_host_staging_bytes(10, 65, 2) == 0
+    assert L.lake_mlp_infer_host(None, 0, 0, None, None, None, 0, None) == lake.LAKE_OK
+    assert L.lake_mlp_infer_host(None, 5, 0, None, None, None, 0, None) == lake.LAKE_ERR_INVAL
+    assert L.lake_mlp_infer_host(16, -1, 0, 16, None, None, 0, None) == lake.LAKE_ERR_INVAL
 
 
 def test_id_width_flags_validated_on_host():

@@ -180,3 +180,32 @@ def test_unaligned_input_rows(name, kernel_path):
     ro, rc = oracle.mlp_family(widths, act, blob, x, nthreads=0)
     _check(act, out.cpu().numpy(), cls.cpu().numpy(), ro, rc)
     lake.mlp_unload(5, 0)
+
+
+@pytest.mark.parametrize("pinned", [True, False])
+@pytest.mark.parametrize("n", [1, 100, 5000])
+def test_infer_host_equals_device(pinned, n):
+    """lake_mlp_infer_host: zero-copy (pinned, mapped) and staged (pageable) host buffers
+    give the device path's results bit for bit."""
+    widths, act = SHAPES["kml"]
+    blob = family.weights(widths, 8)
+    lake.mlp_load(6, widths, act, blob, 0)
+    x = family.features(n, widths[0], 31)
+    o, c = _run(6, x)
+    C = widths[-1]
+    if pinned:
+        hx = torch.from_numpy(x).pin_memory()
+        hc = torch.full((n,), -7, dtype=torch.int32).pin_memory()
+        ho = torch.full((n, C), 12345.0, dtype=torch.float32).pin_memory()
+        lake.mlp_infer_host(hx, n, 6, hc, ho)
+        hc, ho = hc.numpy(), ho.numpy()
+    else:
+        hx = np.ascontiguousarray(x)
+        hc = np.full(n, -7, np.int32)
+        ho = np.full((n, C), 12345.0, np.float32)
+        sb = lake.mlp_host_staging_bytes(n, widths[0], C)
+        stg = torch.empty(sb, dtype=torch.uint8, device=DEV)
+        lake.mlp_infer_host(hx, n, 6, hc, ho, stg, sb)
+    assert np.array_equal(hc, c)
+    assert np.array_equal(ho.view(np.uint32), o.view(np.uint32))
+    lake.mlp_unload(6, 0)
