@@ -19,7 +19,7 @@ constexpr int kMaxHiddenLayers = 3;
 constexpr int kF32TileM = 64;       // I/Os per CTA tile
 constexpr int kF32Threads = 256;
 #ifndef LAKE_F32_KC
-#define LAKE_F32_KC 64
+#define LAKE_F32_KC 16  // 2 CTAs per SM fit only with 16-row chunks (64 was best at 1 CTA/SM)
 #endif
 constexpr int kF32KChunk = LAKE_F32_KC;  // rows of W^T staged per pipeline stage
 constexpr int kF32ActStride = 68;   // floats per activation row in SMEM (64 + 4 pad)

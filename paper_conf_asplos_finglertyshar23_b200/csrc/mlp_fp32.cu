@@ -13,8 +13,8 @@
 // Each accumulator is summed over k strictly in order (that is what a K-loop GEMM does),
 // so the tiling changes nothing numerically. Activations live transposed in SMEM
 // (act[k][row], row stride 68 floats: broadcast A reads, conflict-free epilogue stores);
-// weights stream through a 2-stage cp.async pipeline in 64-row chunks of W^T (16 for the
-// 16-row latency tile), activations are updated in place, and W^T columns
+// weights stream through a 2-stage cp.async pipeline in 16-row chunks of W^T, activations
+// are updated in place (two CTAs fit per SM: 16 warps), and W^T columns
 // were permuted at load time so each thread's 8 columns are two float4s.
 // The 2-wide output layer is one sequential fmaf chain per (row, class).
 #include <cuda_pipeline.h>
@@ -32,7 +32,10 @@ constexpr int kF32Unroll = LAKE_F32_UNROLL;  // k-loop unroll of the RM = 8 tile
 #ifndef LAKE_F32_ACT_BUFS
 #define LAKE_F32_ACT_BUFS 1
 #endif
-constexpr int kF32ActBufs = LAKE_F32_ACT_BUFS;  // 1: in place (frees SMEM for KC = 64)
+constexpr int kF32ActBufs = LAKE_F32_ACT_BUFS;
+#ifndef LAKE_F32_CTAS
+#define LAKE_F32_CTAS 2  // CTAs per SM (<= 128 registers; A/B: 1 -> 2 CTAs +3% NN+2, +36% NN)
+#endif  // 1: in place (frees SMEM for KC = 64)
 
 template <int RM>
 struct F32Cfg {
@@ -41,8 +44,8 @@ struct F32Cfg {
   // activation row stride: float4-aligned with a 4-float pad for RM = 8 (conflict-free
   // float4 epilogue stores), odd for RM = 2 (conflict-free scalar stores)
   static constexpr int S = RM == 8 ? kF32ActStride : M + 1;
-  // rows of W^T per pipeline stage: 64 for the throughput tile (4 syncs per 256-wide layer;
-  // A/B on B200: 16 -> 64 rows +6% on NN+2), 16 for the 16-row latency tile
+  // rows of W^T per pipeline stage (LAKE_F32_KC): 16 so that two CTAs fit per SM (A/B on
+  // B200: 1 CTA/SM with 64-row chunks 6.37 ms, 2 CTAs/SM with 16-row chunks 6.19 ms, C3 NN+2)
   static constexpr int KC = RM == 8 ? kF32KChunk : 16;
 };
 
@@ -68,7 +71,7 @@ __device__ __forceinline__ void stage_chunk(float (*dst)[kHidden], const float *
 }
 
 template <int IN_KIND, int RM>
-__global__ void __launch_bounds__(kF32Threads, 1)
+__global__ void __launch_bounds__(kF32Threads, LAKE_F32_CTAS)
 mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
                 uint8_t *__restrict__ decisions,
                 float *__restrict__ logits) {
@@ -254,7 +257,8 @@ cudaError_t launch_mlp_fp32(const void *in, int in_kind, const TileSched &ts_in,
   // small single-model batches: 16-row tiles (4x less work per tile on the critical path)
   const bool small = ts.tile_model == nullptr && ts.n <= (int64_t)16 * sms;
   if (small) ts.n_tiles = (ts.n + 15) / 16;
-  const int64_t grid = ts.n_tiles < sms ? ts.n_tiles : sms;
+  const int64_t cap = (int64_t)sms * LAKE_F32_CTAS;  // resident CTAs
+  const int64_t grid = ts.n_tiles < cap ? ts.n_tiles : cap;
   if (grid <= 0) return cudaSuccess;
   cudaError_t e;
   if (in_kind == LAKE_IN_RAW)
