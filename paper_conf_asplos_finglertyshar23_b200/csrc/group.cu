@@ -63,19 +63,29 @@ __device__ __forceinline__ bool known(const DevModel *table, int32_t m) {
   return m >= 0 && m < LAKE_MAX_MODELS && table[m].arch >= 0;
 }
 
+// Per-block SMEM copy of "model slot is loaded" so the per-I/O test is a shared-memory byte
+// read instead of a dependent global load of the model table.
+__device__ __forceinline__ void load_known(const DevModel *table, uint8_t *known_s) {
+  for (int m = threadIdx.x; m < LAKE_MAX_MODELS; m += blockDim.x)
+    known_s[m] = table[m].arch >= 0 ? 1 : 0;
+}
+__device__ __forceinline__ int32_t bin_of(const uint8_t *known_s, int32_t m) {
+  return ((unsigned)m < (unsigned)LAKE_MAX_MODELS && known_s[m]) ? m : LAKE_MAX_MODELS;
+}
+
 template <typename IdT>
 __global__ void __launch_bounds__(kGBlock)
 group_hist(const IdT *__restrict__ ids, int64_t n, const DevModel *__restrict__ table,
            WsHeader *h) {
   __shared__ int32_t cnt[LAKE_MAX_MODELS + 1];
+  __shared__ uint8_t known_s[LAKE_MAX_MODELS];
+  load_known(table, known_s);
   for (int64_t base = (int64_t)blockIdx.x * kChunk; base < n; base += (int64_t)gridDim.x * kChunk) {
     for (int i = threadIdx.x; i <= LAKE_MAX_MODELS; i += kGBlock) cnt[i] = 0;
     __syncthreads();
     const int64_t end = (base + kChunk) < n ? base + kChunk : n;
-    for (int64_t i = base + threadIdx.x; i < end; i += kGBlock) {
-      const int32_t m = (int32_t)__ldg(ids + i);
-      atomicAdd(&cnt[known(table, m) ? m : LAKE_MAX_MODELS], 1);
-    }
+    for (int64_t i = base + threadIdx.x; i < end; i += kGBlock)
+      atomicAdd(&cnt[bin_of(known_s, (int32_t)__ldg(ids + i))], 1);
     __syncthreads();
     for (int m = threadIdx.x; m < LAKE_MAX_MODELS; m += kGBlock)
       if (cnt[m]) atomicAdd(&h->counts[m], cnt[m]);
@@ -143,14 +153,14 @@ group_scatter(const IdT *__restrict__ ids, int64_t n, const DevModel *__restrict
               WsHeader *h, int32_t *__restrict__ perm) {
   __shared__ int32_t cnt[LAKE_MAX_MODELS + 1];
   __shared__ int32_t basep[LAKE_MAX_MODELS + 1];
+  __shared__ uint8_t known_s[LAKE_MAX_MODELS];
+  load_known(table, known_s);
   for (int64_t base = (int64_t)blockIdx.x * kChunk; base < n; base += (int64_t)gridDim.x * kChunk) {
     for (int i = threadIdx.x; i <= LAKE_MAX_MODELS; i += kGBlock) cnt[i] = 0;
     __syncthreads();
     const int64_t end = (base + kChunk) < n ? base + kChunk : n;
-    for (int64_t i = base + threadIdx.x; i < end; i += kGBlock) {
-      const int32_t m = (int32_t)__ldg(ids + i);
-      atomicAdd(&cnt[known(table, m) ? m : LAKE_MAX_MODELS], 1);
-    }
+    for (int64_t i = base + threadIdx.x; i < end; i += kGBlock)
+      atomicAdd(&cnt[bin_of(known_s, (int32_t)__ldg(ids + i))], 1);
     __syncthreads();
     for (int m = threadIdx.x; m <= LAKE_MAX_MODELS; m += kGBlock) {
       const int32_t c = cnt[m];
@@ -159,8 +169,7 @@ group_scatter(const IdT *__restrict__ ids, int64_t n, const DevModel *__restrict
     }
     __syncthreads();
     for (int64_t i = base + threadIdx.x; i < end; i += kGBlock) {
-      const int32_t m0 = (int32_t)__ldg(ids + i);
-      const int32_t m = known(table, m0) ? m0 : LAKE_MAX_MODELS;
+      const int32_t m = bin_of(known_s, (int32_t)__ldg(ids + i));
       const int32_t r = atomicAdd(&cnt[m], 1);
       perm[basep[m] + r] = (int32_t)i;
     }
