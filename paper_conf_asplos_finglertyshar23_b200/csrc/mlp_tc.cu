@@ -558,6 +558,21 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         for (int i = 0; i < 16; ++i) w[i] = 0;
         if (valid[half]) {
           if (IN_KIND == LAKE_IN_RAW) {
+#ifndef LAKE_DIG_I2F
+            // Digit pairs converted with packed arithmetic: the 16-bit pattern M | d is the
+            // value M' + d (fp16: 0x6400 = 1024, ulp 1 on [1024, 2048); bf16: 0x4300 = 128,
+            // ulp 1 on [128, 256)), so one packed subtract of (M', M') yields (d0, d1)
+            // exactly for digits 0..9 - about half the instructions of per-digit I2F + packing
+            uint32_t dg[32];
+            digitize_record(rec[half], [&](int k, uint32_t v) { dg[k] = v; });
+            dg[31] = 0;
+            constexpr uint32_t kMagic2 = PREC == 0 ? 0x64006400u : 0x43004300u;
+#pragma unroll
+            for (int pp = 0; pp < 16; ++pp) {
+              const uint32_t u = dg[2 * pp] | (dg[2 * pp + 1] << 16) | kMagic2;
+              w[pp] = PREC == 0 ? ptx::sub_f16x2(u, kMagic2) : ptx::sub_bf16x2(u, kMagic2);
+            }
+#else
             // digit values 0..9 are exact in fp16 and bf16
             digitize_record(rec[half], [&](int k, uint32_t dg) {
               // one integer -> fp16 / bf16 conversion (I2F.F16): 0..9 are exact in both
@@ -565,6 +580,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
                                                : __bfloat16_as_ushort(__uint2bfloat16_rn(dg));
               w[k >> 1] |= (uint32_t)hbits << ((k & 1) * 16);
             });
+#endif
           } else {
 #pragma unroll
             for (int k = 0; k < 31; ++k) {
