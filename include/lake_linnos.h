@@ -168,8 +168,10 @@ int lake_linnos_infer(const void *in, uint32_t flags, int64_t n, int32_t model_i
 size_t lake_linnos_workspace_bytes(int64_t n);
 
 /* Batch scoring across several per-device models in one call (one registry per block
- * device): I/O i is scored with model model_ids[i] (device int32_t[n]).
- * Groups I/Os by model on the device (histogram, scan, stable scatter of indices), then
+ * device): I/O i is scored with model model_ids[i] (device array of n elements
+ * of the type flags & LAKE_IDS_MASK selects: int32_t by default, uint16_t, uint8_t).
+ * Groups I/Os by model on the device (histogram, scan, scatter of indices; the order inside
+ * a model's group is not preserved and does not affect any result), then
  * runs the fused kernel over model-homogeneous tiles and scatters results back to the
  * caller's order. Results equal per-model lake_linnos_infer calls bit for bit.
  * workspace: device buffer of at least lake_linnos_workspace_bytes(n) bytes (else
@@ -204,7 +206,11 @@ int lake_linnos_multi_status(const void *workspace, size_t ws_bytes, int64_t *n_
  * chunk slots). LAKE_PREC_AUTO is resolved once for the whole batch. Batches of at most
  * 2^14 I/Os whose host buffers are all pinned and mapped (cudaHostAlloc / cudaHostRegister
  * under UVA) skip the copies: the kernel reads and writes host memory directly (zero-copy),
- * which is what bounds small-batch latency (Fig. 8's batch sizes). */
+ * which is what bounds small-batch latency (Fig. 8's batch sizes).
+ * h_model_ids holds n elements of the type flags & LAKE_IDS_MASK selects (int32_t by
+ * default, uint16_t or uint8_t; the pointer type is nominal): the upload is PCIe-bound, so
+ * one-byte ids move 37 instead of 40 bytes per I/O. infer_multi reads its device
+ * model_ids the same way. */
 size_t lake_linnos_host_staging_bytes(int64_t n, uint32_t flags);
 int lake_linnos_infer_host(const void *h_in, uint32_t flags, int64_t n, int32_t model_id,
                            const int32_t *h_model_ids, uint8_t *h_decisions, float *h_logits,
