@@ -3,10 +3,11 @@
 // devices arrive interleaved and are scored per model (score_features).
 //
 // Counting sort of I/O indices by model id, on the device:
-//   group_hist     per-block SMEM histogram -> one global atomic per (block, model)
+//   group_hist     per-chunk SMEM histogram -> one global atomic per (chunk, model), and the
+//                  chunk histogram stored for the scatter
 //   group_scan     one block: exclusive scans of counts and of tiles per model (for both
 //                  the 64-row FP32 tiles and the 256-row tensor-core tiles)
-//   group_scatter  per-block SMEM histogram -> reserve a range per model -> positions
+//   group_scatter  stored chunk histogram -> reserve a range per model -> positions
 //   group_tiles    one thread per tile: binary search of its model, begin, count
 // Unknown ids (out of range or not loaded) go to the tail of perm; lake_linnos_multi_grouped
 // writes decision 0 / NaN logits for them. Results do not depend on the order inside a
@@ -18,6 +19,7 @@ namespace {
 
 constexpr int kGBlock = 512;
 constexpr int kChunk = 8192;  // I/Os per block-iteration in hist/scatter
+constexpr int kBins = LAKE_MAX_MODELS + 1;  // model slots + "unknown"
 
 struct WsHeader {
   int32_t counts[LAKE_MAX_MODELS];
@@ -38,7 +40,7 @@ __host__ __device__ inline size_t align256(size_t x) { return (x + 255) & ~(size
 
 struct WsLayout {
   size_t header, perm, t64_model, t64_begin, t64_count, t256_model, t256_begin, t256_count,
-      total;
+      chunk_counts, total;
   int64_t max64, max256;
 };
 
@@ -55,6 +57,8 @@ WsLayout ws_layout(int64_t n) {
   L.t256_model = off; off = align256(off + (size_t)L.max256 * 4);
   L.t256_begin = off; off = align256(off + (size_t)L.max256 * 8);
   L.t256_count = off; off = align256(off + (size_t)L.max256 * 4);
+  // per-chunk histograms written by group_hist, read back by group_scatter (no recount)
+  L.chunk_counts = off; off = align256(off + (size_t)((n + kChunk - 1) / kChunk) * kBins * 4);
   L.total = off;
   return L;
 }
@@ -76,7 +80,7 @@ __device__ __forceinline__ int32_t bin_of(const uint8_t *known_s, int32_t m) {
 template <typename IdT>
 __global__ void __launch_bounds__(kGBlock)
 group_hist(const IdT *__restrict__ ids, int64_t n, const DevModel *__restrict__ table,
-           WsHeader *h) {
+           WsHeader *h, int32_t *__restrict__ chunk_counts) {
   __shared__ int32_t cnt[LAKE_MAX_MODELS + 1];
   __shared__ uint8_t known_s[LAKE_MAX_MODELS];
   load_known(table, known_s);
@@ -87,6 +91,8 @@ group_hist(const IdT *__restrict__ ids, int64_t n, const DevModel *__restrict__ 
     for (int64_t i = base + threadIdx.x; i < end; i += kGBlock)
       atomicAdd(&cnt[bin_of(known_s, (int32_t)__ldg(ids + i))], 1);
     __syncthreads();
+    int32_t *cc = chunk_counts + (base / kChunk) * kBins;
+    for (int m = threadIdx.x; m < kBins; m += kGBlock) cc[m] = cnt[m];
     for (int m = threadIdx.x; m < LAKE_MAX_MODELS; m += kGBlock)
       if (cnt[m]) atomicAdd(&h->counts[m], cnt[m]);
     if (threadIdx.x == 0 && cnt[LAKE_MAX_MODELS])
@@ -150,18 +156,16 @@ group_scan(WsHeader *h) {
 template <typename IdT>
 __global__ void __launch_bounds__(kGBlock)
 group_scatter(const IdT *__restrict__ ids, int64_t n, const DevModel *__restrict__ table,
-              WsHeader *h, int32_t *__restrict__ perm) {
+              WsHeader *h, int32_t *__restrict__ perm, const int32_t *__restrict__ chunk_counts) {
   __shared__ int32_t cnt[LAKE_MAX_MODELS + 1];
   __shared__ int32_t basep[LAKE_MAX_MODELS + 1];
   __shared__ uint8_t known_s[LAKE_MAX_MODELS];
   load_known(table, known_s);
   for (int64_t base = (int64_t)blockIdx.x * kChunk; base < n; base += (int64_t)gridDim.x * kChunk) {
-    for (int i = threadIdx.x; i <= LAKE_MAX_MODELS; i += kGBlock) cnt[i] = 0;
+    const int32_t *cc = chunk_counts + (base / kChunk) * kBins;  // this chunk's histogram
+    for (int i = threadIdx.x; i < kBins; i += kGBlock) cnt[i] = cc[i];
     __syncthreads();
     const int64_t end = (base + kChunk) < n ? base + kChunk : n;
-    for (int64_t i = base + threadIdx.x; i < end; i += kGBlock)
-      atomicAdd(&cnt[bin_of(known_s, (int32_t)__ldg(ids + i))], 1);
-    __syncthreads();
     for (int m = threadIdx.x; m <= LAKE_MAX_MODELS; m += kGBlock) {
       const int32_t c = cnt[m];
       if (c) basep[m] = atomicAdd(m < LAKE_MAX_MODELS ? &h->cursor[m] : &h->unk_cursor, c);
@@ -250,6 +254,7 @@ struct GroupPtrs {
   int32_t *tc[2];
   int32_t *nt[2];
   int64_t max[2];
+  int32_t *cc;  // per-chunk histograms
 };
 
 static GroupPtrs group_ptrs(void *ws, int64_t n) {
@@ -264,6 +269,7 @@ static GroupPtrs group_ptrs(void *ws, int64_t n) {
   p.tm[1] = reinterpret_cast<int32_t *>(b + L.t256_model);
   p.tb[1] = reinterpret_cast<int64_t *>(b + L.t256_begin);
   p.tc[1] = reinterpret_cast<int32_t *>(b + L.t256_count);
+  p.cc = reinterpret_cast<int32_t *>(b + L.chunk_counts);
   p.nt[0] = &p.h->n_tiles64;
   p.nt[1] = &p.h->n_tiles256;
   p.max[0] = L.max64;
@@ -282,10 +288,10 @@ cudaError_t launch_group(int64_t n, const void *model_ids, int id_kind, const De
   const int64_t chunks = (n + kChunk - 1) / kChunk;
   const int grid = (int)(chunks < 2 * sms ? chunks : 2 * sms);
   auto hist = [&](auto *ids) {
-    if (grid > 0) group_hist<<<grid, kGBlock, 0, s>>>(ids, n, table, p.h);
+    if (grid > 0) group_hist<<<grid, kGBlock, 0, s>>>(ids, n, table, p.h, p.cc);
   };
   auto scatter = [&](auto *ids) {
-    if (grid > 0) group_scatter<<<grid, kGBlock, 0, s>>>(ids, n, table, p.h, p.perm);
+    if (grid > 0) group_scatter<<<grid, kGBlock, 0, s>>>(ids, n, table, p.h, p.perm, p.cc);
   };
   const int32_t *i32 = static_cast<const int32_t *>(model_ids);
   const uint16_t *u16 = static_cast<const uint16_t *>(model_ids);
