@@ -26,7 +26,7 @@ namespace lake {
 namespace {
 
 #ifndef LAKE_F32_UNROLL
-#define LAKE_F32_UNROLL 4
+#define LAKE_F32_UNROLL 2  // no register spill at 2 CTAs/SM (4: 32-B spill, same speed)
 #endif
 constexpr int kF32Unroll = LAKE_F32_UNROLL;  // k-loop unroll of the RM = 8 tile
 #ifndef LAKE_F32_ACT_BUFS
