@@ -60,3 +60,33 @@ def test_multi_nn_equals_per_model(prec):
         assert np.array_equal(dec[idx], sdec)
         assert np.array_equal(lg[idx].view(np.uint32), slg.view(np.uint32))
     assert np.all(dec[ids == 5] == 0)
+
+
+@pytest.mark.parametrize("prec", [lake.LAKE_PREC_F16, lake.LAKE_PREC_FP32])
+def test_many_tiny_model_groups(prec):
+    """250 NN+2 models with a skewed I/O count (many groups of 1-3 I/Os): almost every tile
+    of every CTA pair switches model (weight-reload protocol at its densest), plus unknown
+    ids; grouped results equal the oracle per model."""
+    mids = list(range(500, 750))
+    blobs = {m: inputs.weights(2, m) for m in mids}
+    for m in mids:
+        lake.load_weights(m, 2, blobs[m], 0)
+    try:
+        rng = np.random.default_rng(17)
+        p = 1.0 / np.arange(1, len(mids) + 1) ** 1.5
+        ids = np.array(mids)[rng.choice(len(mids), size=30000, p=p / p.sum())].astype(np.int32)
+        ids[::501] = 9999
+        raw = inputs.device_trace("azure", ids.size, 23, rerate=3.0)["raw"]
+        lg, dec, unk = run_multi(raw, ids, lake.LAKE_IN_RAW | prec)
+        assert unk == int((ids == 9999).sum())
+        rlg, rdec = oracle.infer_multi_raw({m: (2, blobs[m]) for m in mids}, raw, ids, nthreads=0)
+        ok = ids != 9999
+        if prec == lake.LAKE_PREC_FP32:
+            assert np.array_equal(dec, rdec)
+            assert np.array_equal(lg[ok].view(np.uint32), rlg[ok].view(np.uint32))
+        else:
+            _check(lg[ok], dec[ok], rlg[ok], rdec[ok])
+            assert np.all(dec[~ok] == 0)
+    finally:
+        for m in mids:
+            lake.unload(m, 0)
