@@ -23,6 +23,7 @@ SHAPES = {
     "w64_relu": ((64, 64, 64, 64, 3), family.ACT_RELU),
     "w1_relu": ((1, 1, 2), family.ACT_RELU),
     "even_in": ((16, 8, 5), family.ACT_RELU),
+    "c64_sig": ((7, 33, 64), family.ACT_SIGMOID),  # widest output layer, odd hidden width
 }
 
 
