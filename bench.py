@@ -50,7 +50,7 @@ def parse():
     p.add_argument("--warmup", type=int, default=5)
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--config", default="C5", choices=["C1", "C3", "C4", "C5"])
-    p.add_argument("--prec", default=None, choices=["fp32", "f16", "bf16"])
+    p.add_argument("--prec", default=None, choices=["fp32", "f16", "bf16", "tf32"])
     p.add_argument("--arch", type=int, default=None)
     p.add_argument("--n-ios", dest="n", type=int, default=None)
     p.add_argument("--mode", default="throughput", choices=["throughput", "sweep", "report", "family"])
@@ -189,7 +189,8 @@ def config_obj(args, wl, prec, world, copies):
                      + (", sharded across ranks (strong scaling)" if world > 1 else "")),
         "n_ios": n, "models": wl["n_models"], "arch": ARCH_NAME[wl["arch"]],
         "path": {"fp32": "CUDA-core FP32 (bit-exact)", "f16": "tcgen05 cta_group::2, fp16 in / fp32 acc",
-                 "bf16": "tcgen05 cta_group::2, bf16 in / fp32 acc"}[prec],
+                 "bf16": "tcgen05 cta_group::2, bf16 in / fp32 acc",
+                 "tf32": "tcgen05 cta_group::2 kind::tf32, tf32 in / fp32 acc"}[prec],
         "input": "raw records (36 B/IO), digitised in-kernel; decisions out (1 B/IO)",
         "api": "lake_linnos_infer_multi (group + fused MLP)",
         "plan": wl["plan"], "imbalance": round(wl["imbalance"], 4),
@@ -296,6 +297,8 @@ def run_ours(args):
         src = "measured (MEASURED_PEAKS.json bf16 burst; fp16:bf16 nominal ratio 1:1)"
         if peak is None:
             peak, src = 1590.0, "fallback (B200_PROFILING.md)"
+        if prec == "tf32":
+            peak, src = peak / 2, src.replace("fp16:bf16 nominal ratio 1:1", "x tf32:bf16 nominal ratio 1:2")
         bound = "tensor"
     flops_launch = ARCH_FLOPS[wl["arch"]] * n_max
     achieved = flops_launch / (kern_avg_max / 1e3) / 1e12
@@ -439,7 +442,7 @@ def run_sweep(args):
     for arch in (0, 1, 2):
         blob = inputs.weights(arch, 0)
         lake.load_weights(40 + arch, arch, blob, 0)
-        for prec in ("fp32", "f16", "bf16"):
+        for prec in ("fp32", "f16", "bf16", "tf32"):
             flags = lake.LAKE_IN_RAW | lake.PREC_FLAGS[prec]
             cross = None
             gcross = None
@@ -561,6 +564,16 @@ def run_report(args):
     fpeak = 148 * 128 * 2 * peaks.get("sm_max_mhz", 1965.0) * 1e6 / 1e12
     rows = []
 
+    def peak_of(prec):
+        return fpeak if prec == "fp32" else (tpeak / 2 if prec == "tf32" else tpeak)
+
+    def peak_label(prec):
+        if prec == "fp32":
+            return "FP32 %.1f TF/s (derived from unit counts)" % fpeak
+        if prec == "tf32":
+            return "tf32 %.1f TF/s = measured bf16 %.1f x nominal tf32:bf16 1:2" % (tpeak / 2, tpeak)
+        return "bf16 %.1f TF/s (measured; fp16 same nominal rate)" % tpeak
+
     def timed(fn, reps=10):
         for _ in range(3):
             fn()
@@ -586,7 +599,7 @@ def run_report(args):
         rlg, rdec = oracle.infer_raw(arch, blob, raw[smp], nthreads=0)
         ref = rlg.astype(np.float64)
         rms = np.sqrt(np.mean(ref ** 2))
-        for prec in ("fp32", "f16", "bf16"):
+        for prec in ("fp32", "f16", "bf16", "tf32"):
             flags = lake.LAKE_IN_RAW | lake.PREC_FLAGS[prec]
             ms = timed(lambda: lake.infer(x, flags, n, 60 + arch, dec, lg, stream))
             lake.infer(x, flags, n, 60 + arch, dec, lg, stream)
@@ -599,9 +612,7 @@ def run_report(args):
             rows.append(dict(config="C3", arch=ARCH_NAME[arch], path=prec, n=n,
                              ms=round(ms, 4), inferences_per_s=round(n / (ms / 1e3), 1),
                              tflops=round(tflops, 2),
-                             frac_of_peak=round(tflops / (fpeak if prec == "fp32" else tpeak), 4),
-                             peak=("FP32 %.1f TF/s (derived)" % fpeak) if prec == "fp32"
-                             else "bf16 %.1f TF/s (measured)" % tpeak,
+                             frac_of_peak=round(tflops / peak_of(prec), 4), peak=peak_label(prec),
                              sample=int(smp.size), agreement=float(1 - dis.mean()),
                              max_rel_err=float(rel.max()),
                              max_disagree_margin=float(np.abs(ref[dis, 0] - ref[dis, 1]).max()) if dis.any() else 0.0,
@@ -657,7 +668,7 @@ def run_report(args):
         rlg[sel], rdec[sel] = oracle.infer_raw(2, w["models"][int(m)][1], w["raw"][smp[sel]], nthreads=0)
     ref = rlg.astype(np.float64)
     rms = np.sqrt(np.mean(ref ** 2))
-    for prec in ("f16", "bf16", "fp32"):
+    for prec in ("f16", "bf16", "tf32", "fp32"):
         flags = lake.LAKE_IN_RAW | lake.PREC_FLAGS[prec]
         ms = timed(lambda: lake.infer_multi(x, flags, n, ids, dec, lg, ws, wsb, stream),
                    reps=10 if prec != "fp32" else 3)
@@ -671,9 +682,7 @@ def run_report(args):
         rows.append(dict(config="C5", arch=ARCH_NAME[2], path=prec, n=n, models=64,
                          ms=round(ms, 4), inferences_per_s=round(n / (ms / 1e3), 1),
                          tflops=round(tflops, 2),
-                         frac_of_peak=round(tflops / (fpeak if prec == "fp32" else tpeak), 4),
-                         peak=("FP32 %.1f TF/s (derived)" % fpeak) if prec == "fp32"
-                         else "bf16 %.1f TF/s (measured)" % tpeak,
+                         frac_of_peak=round(tflops / peak_of(prec), 4), peak=peak_label(prec),
                          api="infer_multi (group + fused MLP), logits written",
                          sample=int(smp.size), agreement=float(1 - dis.mean()),
                          bit_exact_logits=bool(np.array_equal(l.astype(np.float32).view(np.uint32),

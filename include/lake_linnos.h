@@ -101,8 +101,13 @@ enum lake_flags {
     LAKE_PREC_FP32  = 0x00, /* CUDA-core FP32, strict operation order: bit-exact with the
                                oracle (DESIGN.md §3 reading R15)                           */
     LAKE_PREC_F16   = 0x10, /* tcgen05 tensor cores, fp16 operands, fp32 accumulation     */
-    LAKE_PREC_BF16  = 0x20, /* tcgen05 tensor cores, bf16 operands, fp32 accumulation     */
-    LAKE_PREC_TF32  = 0x30, /* reserved: returns LAKE_ERR_UNSUPPORTED (SMEM)   */
+    LAKE_PREC_BF16  = 0x20, /* tcgen05 tensor cores, bf16 operands, fp32 accumulation;
+                               8 mantissa bits: reported, below the north_star agreement
+                               bar on the synthetic models                  */
+    LAKE_PREC_TF32  = 0x30, /* tcgen05 tensor cores (kind::tf32), tf32 operands (fp32
+                               rounded to 10 mantissa bits), fp32 accumulation, half the
+                               fp16 tensor rate; NN+2 streams its last hidden layer's
+                               weights from L2 each tile (272 KB/CTA > SMEM) */
     LAKE_PREC_AUTO  = 0x70, /* FP32 below the model's AUTO threshold, else F16 (below)   */
     LAKE_IDS_I32    = 0x000, /* model_ids: int32_t[n] (default)                         */
     LAKE_IDS_U16    = 0x100, /* model_ids: uint16_t[n]                                   */

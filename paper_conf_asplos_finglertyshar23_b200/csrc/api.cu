@@ -12,6 +12,7 @@
 #include <atomic>
 #include <cmath>
 #include <cstring>
+#include <memory>
 #include <mutex>
 #include <new>
 #include <vector>
@@ -116,46 +117,53 @@ BlobView view_blob(int32_t arch, const float *blob) {
   return v;
 }
 
-// UMMA K-major SWIZZLE_NONE offset (bytes) of element (row r, k) in an R-row operand.
-inline size_t umma_off(int r, int k, int R) {
-  return (size_t)(k >> 3) * (R * 16) + (size_t)r * 16 + (size_t)(k & 7) * 2;
+// UMMA K-major SWIZZLE_NONE offset (bytes) of element (row r, k) in an R-row operand whose
+// elements are `eb` bytes: a core matrix is 8 rows x 16 B (16/eb elements of K).
+inline size_t umma_off(int r, int k, int R, int eb) {
+  const int kc = 16 / eb;  // K elements per core matrix
+  return (size_t)(k / kc) * (R * 16) + (size_t)r * 16 + (size_t)(k % kc) * eb;
 }
 
-template <typename T>
-inline uint16_t to_bits(float v);
-template <>
-inline uint16_t to_bits<__half>(float v) {
-  __half h = __float2half_rn(v);
-  uint16_t u;
-  std::memcpy(&u, &h, 2);
-  return u;
-}
-template <>
-inline uint16_t to_bits<__nv_bfloat16>(float v) {
-  __nv_bfloat16 h = __float2bfloat16_rn(v);
-  uint16_t u;
-  std::memcpy(&u, &h, 2);
-  return u;
+// Operand encodings of one fp32 weight: 0 fp16, 1 bf16 (round to nearest even), 2 tf32
+// (fp32 rounded to nearest even at 10 mantissa bits, low 13 bits zero; finite inputs only,
+// checked at load).
+inline uint32_t to_bits(float v, int prec) {
+  if (prec == 0) {
+    __half h = __float2half_rn(v);
+    uint16_t u;
+    std::memcpy(&u, &h, 2);
+    return u;
+  }
+  if (prec == 1) {
+    __nv_bfloat16 h = __float2bfloat16_rn(v);
+    uint16_t u;
+    std::memcpy(&u, &h, 2);
+    return u;
+  }
+  uint32_t u;
+  std::memcpy(&u, &v, 4);
+  u += 0x0FFFu + ((u >> 13) & 1u);
+  return u & ~0x1FFFu;
 }
 
-template <typename T>
-void build_tc_image(const BlobView &v, uint8_t *img /* 2 * bytes */, size_t bytes) {
+void build_tc_image(const BlobView &v, int prec, uint8_t *img /* 2 * bytes */, size_t bytes) {
   std::memset(img, 0, 2 * bytes);
   const int nh = v.nh;
+  const int eb = (int)tc_elem_bytes(prec);
   for (int rank = 0; rank < 2; ++rank) {
     uint8_t *base = img + rank * bytes;
     auto put = [&](size_t off, float val) {
-      const uint16_t u = to_bits<T>(val);
-      std::memcpy(base + off, &u, 2);
+      const uint32_t u = to_bits(val, prec);
+      std::memcpy(base + off, &u, eb);  // little endian: the low eb bytes
     };
     for (int n = 0; n < 128; ++n)
       for (int k = 0; k < kTcK0; ++k)
-        put(umma_off(n, k, 128), k < 31 ? v.W[0][(size_t)(rank * 128 + n) * 31 + k] : 0.0f);
+        put(umma_off(n, k, 128, eb), k < 31 ? v.W[0][(size_t)(rank * 128 + n) * 31 + k] : 0.0f);
     for (int l = 1; l < nh; ++l) {
-      const size_t o = kTcW0HalfBytes + (size_t)(l - 1) * kTcWhHalfBytes;
+      const size_t o = tc_w0_half_bytes(prec) + (size_t)(l - 1) * tc_wh_half_bytes(prec);
       for (int n = 0; n < 128; ++n)
         for (int k = 0; k < 256; ++k)
-          put(o + umma_off(n, k, 128), v.W[l][(size_t)(rank * 128 + n) * 256 + k]);
+          put(o + umma_off(n, k, 128, eb), v.W[l][(size_t)(rank * 128 + n) * 256 + k]);
     }
   }
 }
@@ -254,7 +262,7 @@ int check_flags(uint32_t flags, int64_t n, int *in_kind, int *prec, int32_t arch
     case LAKE_PREC_FP32: *prec = -1; break;
     case LAKE_PREC_F16: *prec = 0; break;
     case LAKE_PREC_BF16: *prec = 1; break;
-    case LAKE_PREC_TF32: return LAKE_ERR_UNSUPPORTED;
+    case LAKE_PREC_TF32: *prec = 2; break;
     case LAKE_PREC_AUTO: *prec = (n >= auto_min(arch)) ? 0 : -1; break;
     default: return LAKE_ERR_INVAL;
   }
@@ -327,7 +335,8 @@ int lake_linnos_load_weights(int32_t model_id, int32_t arch, const float *blob, 
   // FP32 image: permuted W^T per hidden layer, biases, Wout, bout.
   const size_t f_w0 = 32 * 256, f_wh = 256 * 256;
   const size_t f_total = f_w0 + (nh - 1) * f_wh + nh * 256 + 2 * 256 + 4;
-  std::vector<float> f(f_total, 0.0f);
+  std::unique_ptr<float[]> f(new (std::nothrow) float[f_total]());
+  if (!f) return LAKE_ERR_NOMEM;
   size_t off_wt[kMaxHiddenLayers], off_b[kMaxHiddenLayers], off_wout, off_bout;
   {
     size_t p = 0;
@@ -354,10 +363,15 @@ int lake_linnos_load_weights(int32_t model_id, int32_t arch, const float *blob, 
     f[p] = v.b[nh][0];
     f[p + 1] = v.b[nh][1];
   }
-  const size_t tc_bytes = tc_image_bytes(nh);
-  std::vector<uint8_t> img(4 * tc_bytes);  // [prec][rank]
-  build_tc_image<__half>(v, img.data(), tc_bytes);
-  build_tc_image<__nv_bfloat16>(v, img.data() + 2 * tc_bytes, tc_bytes);
+  // tensor-core images, [prec][rank]: fp16, bf16, tf32
+  size_t tc_off[3], tc_total = 0;
+  for (int p = 0; p < 3; ++p) {
+    tc_off[p] = tc_total;
+    tc_total += 2 * (size_t)tc_image_bytes(nh, p);
+  }
+  std::unique_ptr<uint8_t[]> img(new (std::nothrow) uint8_t[tc_total]);
+  if (!img) return LAKE_ERR_NOMEM;
+  for (int p = 0; p < 3; ++p) build_tc_image(v, p, img.get() + tc_off[p], tc_image_bytes(nh, p));
 
   std::lock_guard<std::mutex> lk(g_mu);
   DeviceGuard dg(device);
@@ -367,12 +381,12 @@ int lake_linnos_load_weights(int32_t model_id, int32_t arch, const float *blob, 
   if (rc != LAKE_OK) return rc;
   ModelBufs nb;
   if (cudaMalloc(&nb.fp32, f_total * 4) != cudaSuccess) return LAKE_ERR_NOMEM;
-  if (cudaMalloc(&nb.tc, img.size()) != cudaSuccess) {
+  if (cudaMalloc(&nb.tc, tc_total) != cudaSuccess) {
     retire_bufs(st, nb);
     return LAKE_ERR_NOMEM;
   }
-  if (cudaMemcpy(nb.fp32, f.data(), f_total * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
-      cudaMemcpy(nb.tc, img.data(), img.size(), cudaMemcpyHostToDevice) != cudaSuccess) {
+  if (cudaMemcpy(nb.fp32, f.get(), f_total * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+      cudaMemcpy(nb.tc, img.get(), tc_total, cudaMemcpyHostToDevice) != cudaSuccess) {
     retire_bufs(st, nb);
     return LAKE_ERR_CUDA;
   }
@@ -380,9 +394,7 @@ int lake_linnos_load_weights(int32_t model_id, int32_t arch, const float *blob, 
   std::memset(&m, 0, sizeof(m));
   m.arch = arch;
   m.nh = nh;
-  m.tc_img[0] = static_cast<const uint8_t *>(nb.tc);
-  m.tc_img[1] = static_cast<const uint8_t *>(nb.tc) + 2 * tc_bytes;
-  m.tc_img_bytes = (uint32_t)tc_bytes;
+  for (int p = 0; p < 3; ++p) m.tc_img[p] = static_cast<const uint8_t *>(nb.tc) + tc_off[p];
   const float *fb = static_cast<const float *>(nb.fp32);
   for (int l = 0; l < nh; ++l) {
     m.wt[l] = fb + off_wt[l];

@@ -32,22 +32,38 @@ constexpr int kF32ActStride = 68;   // floats per activation row in SMEM (64 + 4
 constexpr int kTcRowsPerCta = 128;
 constexpr int kTcTileRows = 256;
 constexpr int kTcK0 = 32;                                   // 31 digits + zero pad
-constexpr uint32_t kTcW0HalfBytes = 128 * kTcK0 * 2;        // 8 KB
-constexpr uint32_t kTcWhHalfBytes = 128 * kHidden * 2;      // 64 KB
-// Per-rank SMEM weight image: W0 half | hidden-layer halves. The biases and the 2-wide
-// output layer stay fp32 (the epilogue stages them from the FP32 image: b[0] .. b[nh-1],
-// W_out[2][256], b_out[2] are contiguous there).
-__host__ __device__ constexpr uint32_t tc_image_bytes(int nh) {
-  return kTcW0HalfBytes + (nh - 1) * kTcWhHalfBytes;
+// Operand element size per precision: prec 0 fp16, 1 bf16 (2 B), 2 tf32 (4 B, fp32 bits
+// with the low 13 mantissa bits zero). A core matrix is 8 rows x 16 B in every case.
+__host__ __device__ constexpr uint32_t tc_elem_bytes(int prec) { return prec == 2 ? 4u : 2u; }
+__host__ __device__ constexpr uint32_t tc_w0_half_bytes(int prec) {
+  return 128u * kTcK0 * tc_elem_bytes(prec);        // 8 KB (16-bit) / 16 KB (tf32)
 }
+__host__ __device__ constexpr uint32_t tc_wh_half_bytes(int prec) {
+  return 128u * kHidden * tc_elem_bytes(prec);      // 64 KB / 128 KB
+}
+constexpr uint32_t kTcW0HalfBytes = tc_w0_half_bytes(0);
+constexpr uint32_t kTcWhHalfBytes = tc_wh_half_bytes(0);
+// Per-rank weight image: W0 half | hidden-layer halves. The biases and the 2-wide output
+// layer stay fp32 (the epilogue stages them from the FP32 image: b[0] .. b[nh-1],
+// W_out[2][256], b_out[2] are contiguous there).
+__host__ __device__ constexpr uint32_t tc_image_bytes(int nh, int prec = 0) {
+  return tc_w0_half_bytes(prec) + (nh - 1) * tc_wh_half_bytes(prec);
+}
+// Bytes of the per-rank image kept resident in SMEM. Everything, except for tf32 NN+2
+// (272 KB per rank > 227 KB): its last hidden layer (W2, 128 KB per rank) is streamed
+// from L2 through an SMEM ring, K-chunk by K-chunk, every tile.
+__host__ __device__ constexpr uint32_t tc_resident_bytes(int nh, int prec) {
+  return (prec == 2 && nh == 3) ? tc_image_bytes(2, 2) : tc_image_bytes(nh, prec);
+}
+constexpr uint32_t kTcRingSlotBytes = 8192;  // tf32 W2 ring slot: 128 rows x K 16
+constexpr uint32_t kTcRingSlots = 4;
 
 struct DevModel {
   int32_t arch;      // -1 = slot empty
   int32_t nh;        // hidden layers: 1, 2, 3
-  // tcgen05 images: [0]=fp16, [1]=bf16; each holds rank-0 half then rank-1 half.
-  const uint8_t *tc_img[2];
-  uint32_t tc_img_bytes;  // bytes per rank half
-  uint32_t pad0;
+  // tcgen05 images: [0]=fp16, [1]=bf16, [2]=tf32; each holds rank-0 half then rank-1 half
+  // (tc_image_bytes(nh, prec) bytes per rank half).
+  const uint8_t *tc_img[3];
   // FP32 path
   const float *wt[kMaxHiddenLayers];  // permuted W^T; layer 0 is [32][256] (row 31 zero)
   const float *b[kMaxHiddenLayers];
@@ -92,7 +108,7 @@ struct GroupView {
   int32_t *counts;
 };
 GroupView group_view(void *ws, int64_t n);
-size_t tc_smem_bytes(int nh_layout);
+size_t tc_smem_bytes(int nh_layout, int prec);
 
 // GPU feature capture (capture.cu)
 size_t capture_workspace_bytes(int64_t n);

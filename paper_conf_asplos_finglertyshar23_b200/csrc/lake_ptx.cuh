@@ -156,6 +156,38 @@ __device__ __forceinline__ void mma_f16_cg2_ts(uint32_t d_tmem, uint32_t a_tmem,
       :: "r"(d_tmem), "r"(a_tmem), "l"(b_desc), "r"(idesc), "r"(accumulate) : "memory");
 }
 
+// kind::tf32 (fp32 storage, 10-bit mantissa operands, fp32 accumulate), CTA pair: A from
+// shared memory / from tensor memory (rows = TMEM lanes, one tf32 per column).
+__device__ __forceinline__ void mma_tf32_cg2(uint32_t d_tmem, uint64_t a_desc, uint64_t b_desc,
+                                             uint32_t idesc, uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::tf32 [%0], %1, %2, %3, p;\n\t}"
+      :: "r"(d_tmem), "l"(a_desc), "l"(b_desc), "r"(idesc), "r"(accumulate) : "memory");
+}
+__device__ __forceinline__ void mma_tf32_cg2_ts(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc,
+                                                uint32_t idesc, uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::tf32 [%0], [%1], %2, %3, p;\n\t}"
+      :: "r"(d_tmem), "r"(a_tmem), "l"(b_desc), "r"(idesc), "r"(accumulate) : "memory");
+}
+// Dispatch on the operand precision (0 fp16, 1 bf16: kind::f16; 2: kind::tf32).
+template <int PREC>
+__device__ __forceinline__ void mma_cg2(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc,
+                                        uint32_t acc) {
+  if constexpr (PREC == 2) mma_tf32_cg2(d, a, b, idesc, acc);
+  else mma_f16_cg2(d, a, b, idesc, acc);
+}
+template <int PREC>
+__device__ __forceinline__ void mma_cg2_ts(uint32_t d, uint32_t a, uint64_t b, uint32_t idesc,
+                                           uint32_t acc) {
+  if constexpr (PREC == 2) mma_tf32_cg2_ts(d, a, b, idesc, acc);
+  else mma_f16_cg2_ts(d, a, b, idesc, acc);
+}
+
 // Arrive (once) on the mbarrier at the same shared offset in every CTA of `cta_mask` when
 // all previously issued tcgen05 async ops of this thread have completed.
 __device__ __forceinline__ void mma_commit_cg2(uint32_t bar, uint16_t cta_mask) {
@@ -240,7 +272,8 @@ __device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint
   return d;
 }
 
-// Instruction descriptor, kind::f16: D fp32, A/B fp16 (fmt 0) or bf16 (fmt 1), both K-major.
+// Instruction descriptor, kind::f16 / kind::tf32: D fp32, A/B fp16 (fmt 0), bf16 (fmt 1) or
+// tf32 (fmt 2, with kind::tf32), both K-major.
 __host__ __device__ constexpr uint32_t umma_idesc_f16(uint32_t ab_fmt, uint32_t M, uint32_t N) {
   return (1u << 4)                 // c_format = F32
          | (ab_fmt << 7)           // a_format
@@ -269,6 +302,14 @@ __device__ __forceinline__ uint32_t pack_f16(float lo, float hi) {
 __device__ __forceinline__ uint32_t pack_bf16(float lo, float hi) {
   uint32_t r;
   asm("cvt.rn.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(hi), "f"(lo));
+  return r;
+}
+
+// ReLU + round-to-nearest-even to tf32 (fp32 bits, low 13 mantissa bits zero): one
+// F2FP.RELU.TF32 instruction.
+__device__ __forceinline__ uint32_t relu_tf32(float v) {
+  uint32_t r;
+  asm("cvt.rn.relu.tf32.f32 %0, %1;" : "=r"(r) : "f"(v));
   return r;
 }
 

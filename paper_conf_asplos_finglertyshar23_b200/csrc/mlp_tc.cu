@@ -37,6 +37,8 @@
 #include <cuda_bf16.h>
 #include <cuda_fp16.h>
 
+#include <atomic>
+
 #include "digitize.cuh"
 #include "lake_internal.h"
 #include "lake_ptx.cuh"
@@ -103,29 +105,38 @@ constexpr uint32_t kEpiCols = kChunkCols / kEpiPerQ;
 constexpr uint32_t kWarpChunks = kChunks;
 constexpr uint32_t kHreadyCount = 2 * kGroupWarps;     // the H group's warps, both CTAs
 #endif
-constexpr uint32_t kKStepsPerChunk = kChunkCols / 16;
+// MMA K per instruction: 16 (fp16/bf16) or 8 (tf32); K-steps per H chunk
+__host__ __device__ constexpr uint32_t kmma(int prec) { return prec == 2 ? 8u : 16u; }
+__host__ __device__ constexpr uint32_t ksteps_per_chunk(int prec) { return kChunkCols / kmma(prec); }
 constexpr int kThreads = 32 * (3 + kEpiWarps + 1);  // digitisers(2) + loader + epi + MMA
 #ifdef LAKE_H_TMEM
 constexpr uint32_t kHBytes = 0;                   // H lives in TMEM
 #else
 constexpr uint32_t kHBytes = 128 * kHidden * 2;   // 64 KB SMEM H tile
 #endif
-constexpr uint32_t kXBytes = 128 * kTcK0 * 2;     // 8 KB
+__host__ __device__ constexpr uint32_t x_bytes(int prec) {  // one X tile, 128 rows x 32
+  return 128u * kTcK0 * tc_elem_bytes(prec);                // 8 KB / 16 KB (tf32)
+}
 constexpr uint32_t kLboR128 = 128 * 16;           // K-direction core stride, 128-row operand
 constexpr uint32_t kPrmFloats = kHidden + 2 * kHidden + 4;  // last-layer bias | W_out | b_out
-constexpr uint32_t kPrm2Words = (kMaxHiddenLayers - 1) * kHidden / 2;  // packed bias pairs
+constexpr uint32_t kPrm2Words = (kMaxHiddenLayers - 1) * kHidden;  // fp32 H-layer biases
 constexpr uint32_t kRedBytes = (kEpiPerQ - 1) * 128 * 2 * 4;  // output-layer partial sums
 
 __host__ __device__ constexpr uint32_t align1k(uint32_t x) { return (x + 1023u) & ~1023u; }
 
+__host__ __device__ constexpr bool streams_w2(int nh, int prec) {
+  return tc_resident_bytes(nh, prec) < tc_image_bytes(nh, prec);
+}
+
 struct Layout {
-  uint32_t h, x, prm, red, prm0, red0, bar, total;
+  uint32_t ring, h, x, prm, red, prm0, red0, bar, total;
 };
-__host__ __device__ constexpr Layout tc_layout(int nh_layout) {
+__host__ __device__ constexpr Layout tc_layout(int nh_layout, int prec) {
   Layout L{};
-  L.h = align1k(tc_image_bytes(nh_layout));
+  L.ring = align1k(tc_resident_bytes(nh_layout, prec));
+  L.h = L.ring + (streams_w2(nh_layout, prec) ? kTcRingSlots * kTcRingSlotBytes : 0u);
   L.x = L.h + kHBytes;
-  L.prm = L.x + 2 * kXBytes;
+  L.prm = L.x + 2 * x_bytes(prec);
   L.red = L.prm + kPrmFloats * 4 + kPrm2Words * 4;
   // group 0's own copy of the output-layer parameters and partial sums: with two epilogue
   // groups, NN tiles (a single layer) are drained by the group of their accumulator buffer
@@ -135,13 +146,19 @@ __host__ __device__ constexpr Layout tc_layout(int nh_layout) {
   L.total = L.bar + 256;
   return L;
 }
+static_assert(tc_layout(3, 2).total <= 232448, "tf32 NN+2 layout exceeds 227 KB");
+static_assert(tc_layout(3, 0).total <= 232448, "fp16 NN+2 layout exceeds 227 KB");
 
 // barrier slots (8 bytes each) inside the barrier block
 enum : uint32_t {
   B_WLOAD = 0, B_WREADY = 1, B_XFULL = 2, B_XEMPTY = 4, B_DFULL = 6, B_DFULLX = 8,
-  B_TEMPTY = 10, B_HREADY = 12, B_WFREE = 12 + kChunks, B_COUNT = 13 + kChunks
+  B_TEMPTY = 10, B_HREADY = 12, B_WFREE = 12 + kChunks,
+  B_RFULL = 13 + kChunks,                 // [kTcRingSlots] W2 ring slot loaded (tf32 NN+2)
+  B_REMPTY = B_RFULL + kTcRingSlots,      // [kTcRingSlots] W2 ring slot consumed
+  B_COUNT = B_REMPTY + kTcRingSlots
 };
 constexpr uint32_t kTmemSlot = B_COUNT * 8;  // u32 TMEM base address
+static_assert(kTmemSlot + 4 <= 256, "barrier block");
 
 // Per-tile schedule entry. Each role loads tile t+1's entry at the top of tile t (the
 // global loads then overlap tile t's work instead of stalling the next iteration).
@@ -186,56 +203,50 @@ constexpr uint32_t kWarpLoad = 3;
 constexpr uint32_t kWarpEpi = 4;
 #endif
 
-__device__ __forceinline__ uint32_t img_w0() { return 0; }
-__device__ __forceinline__ uint32_t img_wh(int l) { return kTcW0HalfBytes + (l - 1) * kTcWhHalfBytes; }
-
-// H chunk epilogue for one warp: 32 rows x 32 columns of fp32 accumulator -> packed
-// fp16/bf16 pairs -> + bias, ReLU (one packed FMA per pair) -> H (K-major core layout).
-// bias2 holds the layer's biases as packed pairs in the operand type.
-template <int PREC, int W>
-__device__ __forceinline__ void epi_to_h(const uint32_t (&r)[W], const uint32_t *bias2,
-                                         uint32_t col0, uint32_t hrow_addr) {
-  const uint32_t one2 = PREC == 0 ? 0x3C003C00u : 0x3F803F80u;
-#pragma unroll
-  for (int gq = 0; gq < W / 8; ++gq) {
-    const uint4 bb = *reinterpret_cast<const uint4 *>(bias2 + (col0 >> 1) + gq * 4);
-    const uint32_t bv[4] = {bb.x, bb.y, bb.z, bb.w};
-    uint32_t p[4];
-#pragma unroll
-    for (int e = 0; e < 4; ++e) {
-      const int c = gq * 8 + e * 2;
-      const float v0 = __uint_as_float(r[c]), v1 = __uint_as_float(r[c + 1]);
-      if (PREC == 0)
-        p[e] = ptx::hfma2_relu_f16(ptx::pack_f16(v0, v1), one2, bv[e]);
-      else
-        p[e] = ptx::hfma2_relu_bf16(ptx::pack_bf16(v0, v1), one2, bv[e]);
-    }
-    ptx::st_shared_v4(hrow_addr + ((col0 >> 3) + gq) * kLboR128, p[0], p[1], p[2], p[3]);
-  }
+__device__ __forceinline__ uint32_t img_wh(int l, int prec) {
+  return tc_w0_half_bytes(prec) + (l - 1) * tc_wh_half_bytes(prec);
 }
 
-// Same conversion, but the packed pairs go back into tensor memory, in place: the warp's
-// own W fp32 columns [col0, col0+W) (just read) become W/2 packed columns [col0, col0+W/2),
-// which the next layer's MMA reads as its A operand (H kept in TMEM, no SMEM / proxy fence).
-// K-step s (features 16s..16s+15) therefore sits at packed column tmem_a_col(s).
+// Column of TMEM (relative to the H buffer) where K-step s of the next layer's A operand
+// sits. fp16/bf16: the warp's kEpiCols fp32 columns [col0, col0 + kEpiCols) are packed in
+// place into kEpiCols/2 columns [col0, col0 + kEpiCols/2), so K-step s (features 16s..16s+15)
+// is at packed column tmem_a_col(s). tf32: one value per column, in place: column 8s.
+template <int PREC>
+__host__ __device__ constexpr uint32_t tmem_a_col(uint32_t s) {
+  if constexpr (PREC == 2) return s * 8;
+  else return (s / (kEpiCols / 16)) * kEpiCols + (s % (kEpiCols / 16)) * 8;
+}
+
+// H chunk epilogue for one warp (H kept in TMEM): W fp32 accumulator columns of its 32 rows
+// -> + bias (fp32, one rounding) -> ReLU + one rounding to the operand type -> written back
+// in place into the accumulator it came from (see tmem_a_col), where the next layer's MMA
+// reads it as its A operand (no SMEM H tile, no proxy fence).
 template <int PREC, int W>
-__device__ __forceinline__ void epi_to_h_tmem(const uint32_t (&r)[W], const uint32_t *bias2,
+__device__ __forceinline__ void epi_to_h_tmem(const uint32_t (&r)[W], const float *bias,
                                               uint32_t col0, uint32_t tlane_base) {
-  const uint32_t one2 = PREC == 0 ? 0x3C003C00u : 0x3F803F80u;
-  uint32_t p[W / 2];
+  constexpr int NW = PREC == 2 ? W : W / 2;  // 32-bit words written back
+  uint32_t p[NW];
 #pragma unroll
-  for (int gq = 0; gq < W / 8; ++gq) {
-    const uint4 bb = *reinterpret_cast<const uint4 *>(bias2 + (col0 >> 1) + gq * 4);
-    const uint32_t bv[4] = {bb.x, bb.y, bb.z, bb.w};
+  for (int c4 = 0; c4 < W / 4; ++c4) {
+    const float4 b4 = *reinterpret_cast<const float4 *>(bias + col0 + c4 * 4);
+    const float bb[4] = {b4.x, b4.y, b4.z, b4.w};
 #pragma unroll
-    for (int e = 0; e < 4; ++e) {
-      const int c = gq * 8 + e * 2;
-      const float v0 = __uint_as_float(r[c]), v1 = __uint_as_float(r[c + 1]);
+    for (int e = 0; e < 4; e += 2) {
+      const int c = c4 * 4 + e;
 #ifdef LAKE_ABL_NOCVT  // timing-only ablation: no conversion arithmetic
-      p[gq * 4 + e] = r[c] ^ r[c + 1] ^ bv[e];
+      if constexpr (PREC == 2) { p[c] = r[c]; p[c + 1] = r[c + 1]; }
+      else p[c / 2] = r[c] ^ r[c + 1];
 #else
-      p[gq * 4 + e] = PREC == 0 ? ptx::hfma2_relu_f16(ptx::pack_f16(v0, v1), one2, bv[e])
-                                : ptx::hfma2_relu_bf16(ptx::pack_bf16(v0, v1), one2, bv[e]);
+      const float v0 = __uint_as_float(r[c]) + bb[e];
+      const float v1 = __uint_as_float(r[c + 1]) + bb[e + 1];
+      if constexpr (PREC == 2) {
+        p[c] = ptx::relu_tf32(v0);
+        p[c + 1] = ptx::relu_tf32(v1);
+      } else if constexpr (PREC == 0) {
+        p[c / 2] = ptx::relu_pack_f16(v0, v1);
+      } else {
+        p[c / 2] = ptx::relu_pack_bf16(v0, v1);
+      }
 #endif
     }
   }
@@ -243,13 +254,9 @@ __device__ __forceinline__ void epi_to_h_tmem(const uint32_t (&r)[W], const uint
   if (p[0] == 0x12345678u && p[1] == 0x9abcdef0u)
 #endif
   {
-    if constexpr (W / 2 == 16) ptx::tmem_st_32x32b_x16(tlane_base + col0, p);
+    if constexpr (NW == 16) ptx::tmem_st_32x32b_x16(tlane_base + col0, p);
     else ptx::tmem_st_32x32b_x8(tlane_base + col0, p);
   }
-}
-
-__host__ __device__ constexpr uint32_t tmem_a_col(uint32_t s) {
-  return (s / (kEpiCols / 16)) * kEpiCols + (s % (kEpiCols / 16)) * 8;
 }
 
 // Last hidden layer: ReLU(acc + b) in fp32, accumulated straight into the two logits
@@ -284,7 +291,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
 mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts, int nh_layout,
               uint8_t *__restrict__ decisions, float *__restrict__ logits) {
   extern __shared__ __align__(1024) uint8_t smem[];
-  const Layout L = tc_layout(nh_layout);
+  const Layout L = tc_layout(nh_layout, PREC);
+  constexpr uint32_t kXB = x_bytes(PREC);
+  constexpr uint32_t kKS = ksteps_per_chunk(PREC);  // MMA K-steps per H chunk
+  constexpr uint32_t kK0S = kTcK0 / kmma(PREC);       // MMA K-steps of layer 0
   const uint32_t sbase = ptx::smem_u32(smem);
   const uint32_t bar0 = sbase + L.bar;
   auto bar = [&](uint32_t slot) { return bar0 + slot * 8; };
@@ -324,12 +334,14 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       ptx::mbar_init(bar(B_DFULLX + i), 1);      // tcgen05.commit (multicast): last layer
       ptx::mbar_init(bar(B_TEMPTY + i), 2 * kGroupWarps);  // the draining group, both CTAs
     }
-#ifdef LAKE_ABL_LOCALREADY  // timing-only ablation: chunk-ready counts only the leader's warps
-    for (uint32_t i = 0; i < kChunks; ++i) ptx::mbar_init(bar(B_HREADY + i), kHreadyCount / 2);
-#else
     for (uint32_t i = 0; i < kChunks; ++i) ptx::mbar_init(bar(B_HREADY + i), kHreadyCount);
-#endif
     ptx::mbar_init(bar(B_WFREE), 1);             // tcgen05.commit (multicast)
+    for (uint32_t i = 0; i < kTcRingSlots; ++i) {
+      // leader: its own loader's arrive.expect_tx (+ bytes) and the peer's forwarded arrive;
+      // peer: its loader's arrive.expect_tx (+ bytes)
+      ptx::mbar_init(bar(B_RFULL + i), rank == 0 ? 2 : 1);
+      ptx::mbar_init(bar(B_REMPTY + i), 1);      // tcgen05.commit (multicast)
+    }
     ptx::fence_mbar_init();
   }
   if (warp == kWarpLoad) {
@@ -343,34 +355,69 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
 
   if (warp == kWarpLoad) {
     // ================= weight loader (both CTAs) =================
+    // Resident part of the model's image at model switches; for tf32 NN+2 also the W2
+    // K-slices of every tile into the ring (kTcRingSlots x 8 KB, 16 slices per tile).
     if (lane == 0) {
       const uint8_t *cur = nullptr;
       uint32_t wl_phase = 0, wf_phase = 0;
+      uint32_t rc = 0;  // ring slices issued
       const uint32_t wready_leader = ptx::mapa(bar(B_WREADY), 0);
       for (int64_t t = t_begin; t < t_end; ++t) {
         const TileInfo ti = tile_info<PREC>(ts, t);
-        if (ti.img == cur) continue;
-        // Model switch: every MMA reading the old weights must have completed. The MMA
-        // thread commits B_WFREE once per switch, after the old model's last MMA; it cannot
-        // commit the next one before this loader has signalled B_WREADY (lag <= 1 phase).
-        if (cur) {
-          ptx::mbar_wait(bar(B_WFREE), wf_phase);
-          wf_phase ^= 1;
+        const uint8_t *src = ti.img + (size_t)rank * tc_image_bytes(ti.nh, PREC);
+        if (ti.img != cur) {
+          // Model switch: every MMA reading the old weights must have completed. The MMA
+          // thread commits B_WFREE once per switch, after the old model's last MMA; it
+          // cannot commit the next one before this loader has signalled B_WREADY.
+          if (cur) {
+            ptx::mbar_wait(bar(B_WFREE), wf_phase);
+            wf_phase ^= 1;
+          }
+          const uint32_t bytes = tc_resident_bytes(ti.nh, PREC);
+          ptx::mbar_arrive_expect_tx(bar(B_WLOAD), bytes);
+          for (uint32_t off = 0; off < bytes; off += 32768) {
+            const uint32_t len = (bytes - off) < 32768 ? (bytes - off) : 32768;
+            ptx::bulk_g2s(sbase + off, src + off, len, bar(B_WLOAD));
+          }
+          ptx::mbar_wait(bar(B_WLOAD), wl_phase);
+          wl_phase ^= 1;
+          ptx::mbar_arrive_cluster(wready_leader);
+          cur = ti.img;
         }
-        const uint32_t bytes = ti.model->tc_img_bytes;
-        const uint8_t *src = ti.img + (size_t)rank * bytes;
-        ptx::mbar_arrive_expect_tx(bar(B_WLOAD), bytes);
-        for (uint32_t off = 0; off < bytes; off += 32768) {
-          const uint32_t len = (bytes - off) < 32768 ? (bytes - off) : 32768;
-          ptx::bulk_g2s(sbase + off, src + off, len, bar(B_WLOAD));
+        if constexpr (PREC == 2) {
+          if (streams_w2(ti.nh, PREC)) {
+            const uint8_t *w2 = src + img_wh(2, PREC);
+            for (uint32_t c = 0; c < tc_wh_half_bytes(PREC) / kTcRingSlotBytes; ++c, ++rc) {
+              const uint32_t slot = rc % kTcRingSlots;
+              if (rc >= kTcRingSlots)
+                ptx::mbar_wait(bar(B_REMPTY + slot), ((rc / kTcRingSlots) - 1) & 1);
+              ptx::mbar_arrive_expect_tx(bar(B_RFULL + slot), kTcRingSlotBytes);
+              ptx::bulk_g2s(sbase + L.ring + slot * kTcRingSlotBytes, w2 + c * kTcRingSlotBytes,
+                            kTcRingSlotBytes, bar(B_RFULL + slot));
+            }
+          }
         }
-        ptx::mbar_wait(bar(B_WLOAD), wl_phase);
-        wl_phase ^= 1;
-        ptx::mbar_arrive_cluster(wready_leader);
-        cur = ti.img;
       }
     }
   } else if (warp == kWarpMma) {
+    if constexpr (PREC == 2) {
+      // ================= ring forwarder (peer CTA, one thread) =================
+      // The leader's MMA reads both CTAs' W2 halves, but may only wait on its own
+      // mbarriers: forward each completed peer slice to the leader's B_RFULL.
+      if (rank == 1 && lane == 0) {
+        const uint32_t rfull_leader0 = ptx::mapa(bar(B_RFULL), 0);
+        uint32_t fc = 0;
+        for (int64_t t = t_begin; t < t_end; ++t) {
+          const TileInfo ti = tile_info<PREC>(ts, t);
+          if (!streams_w2(ti.nh, PREC)) continue;
+          for (uint32_t c = 0; c < tc_wh_half_bytes(PREC) / kTcRingSlotBytes; ++c, ++fc) {
+            const uint32_t slot = fc % kTcRingSlots;
+            ptx::mbar_wait(bar(B_RFULL + slot), (fc / kTcRingSlots) & 1);
+            ptx::mbar_arrive_cluster(rfull_leader0 + slot * 8);
+          }
+        }
+      }
+    }
     // ================= MMA issuer (leader CTA, one thread) =================
     if (rank == 0 && lane == 0) {
 #ifdef LAKE_ABL_HALFN  // timing-only ablation: hidden-layer MMAs with N = 128 (half the work)
@@ -378,19 +425,21 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
 #else
       const uint32_t idesc = ptx::umma_idesc_f16(PREC, 256, 256);
 #endif
-      // descriptors: advancing K by 16 elements = +2 core matrices = +2*LBO bytes, i.e.
-      // +(2*LBO)>>4 in the 14-bit start-address field (no carry: SMEM < 256 KB)
+      // descriptors: one MMA K-step (16 fp16/bf16 or 8 tf32 = 32 B) = +2 core matrices =
+      // +2*LBO bytes, i.e. +(2*LBO)>>4 in the 14-bit start-address field (no carry: SMEM <
+      // 256 KB)
       constexpr uint64_t kStep = (2 * kLboR128) >> 4;
       const uint64_t xdesc0 = ptx::umma_desc(sbase + L.x, kLboR128, 128);
-      const uint64_t xdesc1 = ptx::umma_desc(sbase + L.x + kXBytes, kLboR128, 128);
-      const uint64_t w0desc = ptx::umma_desc(sbase + img_w0(), kLboR128, 128);
-      const uint64_t hdesc = ptx::umma_desc(sbase + L.h, kLboR128, 128);
+      const uint64_t xdesc1 = ptx::umma_desc(sbase + L.x + kXB, kLboR128, 128);
+      const uint64_t w0desc = ptx::umma_desc(sbase, kLboR128, 128);
+      const uint64_t ringdesc = ptx::umma_desc(sbase + L.ring, kLboR128, 128);
       uint64_t whdesc[kMaxHiddenLayers];
       for (int l = 1; l < kMaxHiddenLayers; ++l)
-        whdesc[l] = ptx::umma_desc(sbase + img_wh(l), kLboR128, 128);
+        whdesc[l] = ptx::umma_desc(sbase + img_wh(l, PREC), kLboR128, 128);
       const uint8_t *cur = nullptr;
       uint32_t w_phase = 0, g = 0, h_phase = 0, t_phase = 0;  // h/t_phase: one bit per slot
       uint32_t used = 0;  // bit b: accumulator b has been written before
+      uint32_t mc = 0;    // ring slices consumed
       int64_t it = 0;
       auto acquire_buf = [&](uint32_t b) {  // accumulator b must be drained by the epilogues
         if (used & (1u << b)) {
@@ -401,18 +450,12 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       };
       TileInfo nxt;
       if (t_begin < t_end) nxt = tile_info<PREC>(ts, t_begin);
-#ifndef LAKE_NO_MMA_SCHED2
-#define LAKE_MMA_SCHED2 1
-#endif
-#ifdef LAKE_MMA_SCHED2
       // schedule entries two tiles ahead: the model slot of tile t+2 is loaded at the top of
       // tile t and the dependent model-table loads of tile t+1 are issued there too, from a
       // slot loaded one tile earlier, so no load result is waited for on the tile boundary
       auto slot_of = [&](int64_t tt) -> int32_t { return ts.tile_model ? ts.tile_model[tt] : -1; };
       int32_t slot_n = (t_begin + 1 < t_end) ? slot_of(t_begin + 1) : -1;
-#endif
       for (int64_t t = t_begin; t < t_end; ++t, ++it) {
-#ifdef LAKE_MMA_SCHED2
         const TileInfo ti = nxt;
         const int32_t slot_nn = (t + 2 < t_end) ? slot_of(t + 2) : -1;
         if (t + 1 < t_end) {
@@ -422,19 +465,13 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           nxt.nh = mm->nh;
         }
         slot_n = slot_nn;
-#elif defined(LAKE_NO_PREFETCH)
-        const TileInfo ti = tile_info<PREC>(ts, t);
-        if (t + 1 < t_end) nxt = tile_info<PREC>(ts, t + 1);
-#else
-        const TileInfo ti = nxt;
-        if (t + 1 < t_end) nxt = tile_info<PREC>(ts, t + 1);
-#endif
         if (ti.img != cur) {
           ptx::mbar_wait(bar(B_WREADY), w_phase);
           w_phase ^= 1;
           cur = ti.img;
         }
         const int nh = ti.nh;
+        const bool stream = streams_w2(nh, PREC);
         const uint32_t xb = (uint32_t)(it & 1);
         {  // layer 0: D = X[128(x2) x 32] * W0^T
           const uint32_t b = g & 1;
@@ -446,8 +483,8 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           const uint32_t d = tmem + b * 256;
           const uint64_t xd = xb ? xdesc1 : xdesc0;
 #pragma unroll
-          for (uint32_t s = 0; s < kTcK0 / 16; ++s)
-            ptx::mma_f16_cg2(d, xd + s * kStep, w0desc + s * kStep, idesc, s);
+          for (uint32_t s = 0; s < kK0S; ++s)
+            ptx::mma_cg2<PREC>(d, xd + s * kStep, w0desc + s * kStep, idesc, s);
           ptx::mma_commit_cg2(bar(B_XEMPTY + xb), 0x3);
           // NN: the accumulator's buffer picks the draining group (b0 -> group 0, b1 -> 1),
           // so both groups convert logits and two NN tiles are drained at once
@@ -462,36 +499,41 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           LAKE_TEV(T_TEMPTY, it, l, 0);
           ptx::tc_fence_after();
           const uint32_t d = tmem + b * 256;
+          // A = H(l-1), in place in the previous layer's accumulator buffer
+          const uint32_t ha = tmem + ((g - 1) & 1) * 256;
+          const bool from_ring = stream && l == 2;
+          const uint64_t wd = l == 1 ? whdesc[1] : whdesc[2];
           for (uint32_t kc = 0; kc < kChunks; ++kc) {
             ptx::mbar_wait(bar(B_HREADY + kc), (h_phase >> kc) & 1);
             h_phase ^= (1u << kc);
             LAKE_TEV(T_HREADY, it, l, kc);
             ptx::tc_fence_after();
-#ifdef LAKE_H_TMEM
-            // A = H(l-1), packed in place in the previous layer's accumulator buffer
-            const uint32_t ha = tmem + ((g - 1) & 1) * 256;
-            const uint64_t wd = l == 1 ? whdesc[1] : whdesc[2];
+            if (from_ring) {
+              // W2 K-slices from the ring: one 8-KB slot = 16 K = 2 tf32 K-steps
+              constexpr uint32_t kSPS = kTcRingSlotBytes / (2 * kLboR128);  // K-steps per slot
 #pragma unroll
-            for (uint32_t s = 0; s < kKStepsPerChunk; ++s) {
-              const uint32_t ks = kc * kKStepsPerChunk + s;
-              ptx::mma_f16_cg2_ts(d, ha + tmem_a_col(ks), wd + ks * kStep, idesc, ks);
-            }
-#elif defined(LAKE_INLINE_DESC)
+              for (uint32_t s = 0; s < kKS; ++s) {
+                const uint32_t ks = kc * kKS + s;
+                const uint32_t slot = mc % kTcRingSlots;
+                if (s % kSPS == 0) {
+                  ptx::mbar_wait(bar(B_RFULL + slot), (mc / kTcRingSlots) & 1);
+                  ptx::tc_fence_after();
+                }
+                ptx::mma_cg2_ts<PREC>(d, ha + tmem_a_col<PREC>(ks),
+                                      ringdesc + (slot * kTcRingSlotBytes >> 4) + (s % kSPS) * kStep,
+                                      idesc, ks);
+                if (s % kSPS == kSPS - 1) {
+                  ptx::mma_commit_cg2(bar(B_REMPTY + slot), 0x3);
+                  ++mc;
+                }
+              }
+            } else {
 #pragma unroll
-            for (uint32_t s = 0; s < kKStepsPerChunk; ++s) {
-              const uint32_t ks = kc * kKStepsPerChunk + s;
-              ptx::mma_f16_cg2(d, ptx::umma_desc(sbase + L.h + ks * 2 * kLboR128, kLboR128, 128),
-                               ptx::umma_desc(sbase + img_wh(l) + ks * 2 * kLboR128, kLboR128, 128),
-                               idesc, ks);
+              for (uint32_t s = 0; s < kKS; ++s) {
+                const uint32_t ks = kc * kKS + s;
+                ptx::mma_cg2_ts<PREC>(d, ha + tmem_a_col<PREC>(ks), wd + ks * kStep, idesc, ks);
+              }
             }
-#else
-            const uint64_t wd = l == 1 ? whdesc[1] : whdesc[2];
-#pragma unroll
-            for (uint32_t s = 0; s < kKStepsPerChunk; ++s) {
-              const uint32_t ks = kc * kKStepsPerChunk + s;
-              ptx::mma_f16_cg2(d, hdesc + ks * kStep, wd + ks * kStep, idesc, ks);
-            }
-#endif
             LAKE_TEV(T_ISSUED, it, l, kc);
           }
           ptx::mma_commit_cg2(bar((kEpiGroups == 2 && l + 1 == nh ? B_DFULLX : B_DFULL) + b), 0x3);
@@ -503,7 +545,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       }
     }
   } else if (warp >= kWarpDig && warp < kWarpDig + 2) {
-    // ================= digitisers: raw -> X (fp16/bf16 digits), 2 rows per thread ========
+    // ================= digitisers: raw -> X (operand-type digits), 2 rows per thread ======
     // Both rows' gathers are issued before any shared store (the st.shared asm carries a
     // memory clobber, so loads written after it could not be hoisted): the two rows' global
     // latencies overlap.
@@ -549,52 +591,57 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         ptx::mbar_wait(bar(B_XEMPTY + xb), (uint32_t)(((it >> 1) & 1) ^ 1));
         LAKE_TEV(T_XEMPTY, it, 0, 0);
       }
-      const uint32_t xs = sbase + L.x + xb * kXBytes;
+      const uint32_t xs = sbase + L.x + xb * kXB;
 #pragma unroll
       for (int half = 0; half < 2; ++half) {
         const uint32_t r = d + 64 * half;
-        uint32_t w[16];
+        // the row's 32 K values (31 digits + the zero pad) in the operand type
+        uint32_t dg[32];
 #pragma unroll
-        for (int i = 0; i < 16; ++i) w[i] = 0;
+        for (int i = 0; i < 32; ++i) dg[i] = 0;
         if (valid[half]) {
           if (IN_KIND == LAKE_IN_RAW) {
-#ifndef LAKE_DIG_I2F
-            // Digit pairs converted with packed arithmetic: the 16-bit pattern M | d is the
-            // value M' + d (fp16: 0x6400 = 1024, ulp 1 on [1024, 2048); bf16: 0x4300 = 128,
-            // ulp 1 on [128, 256)), so one packed subtract of (M', M') yields (d0, d1)
-            // exactly for digits 0..9 - about half the instructions of per-digit I2F + packing
-            uint32_t dg[32];
             digitize_record(rec[half], [&](int k, uint32_t v) { dg[k] = v; });
-            dg[31] = 0;
-            constexpr uint32_t kMagic2 = PREC == 0 ? 0x64006400u : 0x43004300u;
-#pragma unroll
-            for (int pp = 0; pp < 16; ++pp) {
-              const uint32_t u = dg[2 * pp] | (dg[2 * pp + 1] << 16) | kMagic2;
-              w[pp] = PREC == 0 ? ptx::sub_f16x2(u, kMagic2) : ptx::sub_bf16x2(u, kMagic2);
-            }
-#else
-            // digit values 0..9 are exact in fp16 and bf16
-            digitize_record(rec[half], [&](int k, uint32_t dg) {
-              // one integer -> fp16 / bf16 conversion (I2F.F16): 0..9 are exact in both
-              const uint16_t hbits = PREC == 0 ? __half_as_ushort(__uint2half_rn(dg))
-                                               : __bfloat16_as_ushort(__uint2bfloat16_rn(dg));
-              w[k >> 1] |= (uint32_t)hbits << ((k & 1) * 16);
-            });
-#endif
           } else {
 #pragma unroll
-            for (int k = 0; k < 31; ++k) {
-              const uint32_t v = (rec[half][k >> 2] >> ((k & 3) * 8)) & 0xFFu;  // 0..255: exact
-              const uint16_t hbits = PREC == 0 ? __half_as_ushort(__uint2half_rn(v))
-                                               : __bfloat16_as_ushort(__uint2bfloat16_rn(v));
-              w[k >> 1] |= (uint32_t)hbits << ((k & 1) * 16);
-            }
+            for (int k = 0; k < 31; ++k) dg[k] = (rec[half][k >> 2] >> ((k & 3) * 8)) & 0xFFu;
           }
         }
+        if constexpr (PREC == 2) {
+          // tf32 = fp32 bits: 0x4B000000 | v is the float 2^23 + v, exact for v < 2^23, so
+          // one subtract of 2^23 gives v exactly (digits 0..9, digit bytes 0..255)
+          uint32_t w[32];
 #pragma unroll
-        for (int kg = 0; kg < 4; ++kg)
-          ptx::st_shared_v4(xs + kg * kLboR128 + r * 16, w[kg * 4 + 0], w[kg * 4 + 1],
-                            w[kg * 4 + 2], w[kg * 4 + 3]);
+          for (int k = 0; k < 32; ++k)
+            w[k] = __float_as_uint(__uint_as_float(0x4B000000u | dg[k]) - 8388608.0f);
+#pragma unroll
+          for (int kg = 0; kg < 8; ++kg)
+            ptx::st_shared_v4(xs + kg * kLboR128 + r * 16, w[kg * 4 + 0], w[kg * 4 + 1],
+                              w[kg * 4 + 2], w[kg * 4 + 3]);
+        } else {
+          // Value pairs converted with packed arithmetic: the 16-bit pattern M | v is the
+          // value M' + v (fp16: 0x6400 = 1024, ulp 1 on [1024, 2048); bf16: 0x4300 = 128,
+          // ulp 1 on [128, 256)), so one packed subtract of (M', M') yields (v0, v1) exactly
+          // for v < 128 - about half the instructions of per-value I2F + packing. Digit bytes
+          // of LAKE_IN_DIGITS input can reach 255, exact in fp16 (< 1024) but not by the bf16
+          // trick, so that case converts value by value.
+          uint32_t w[16];
+          constexpr uint32_t kMagic2 = PREC == 0 ? 0x64006400u : 0x43004300u;
+#pragma unroll
+          for (int pp = 0; pp < 16; ++pp) {
+            if (IN_KIND == LAKE_IN_RAW || PREC == 0) {
+              const uint32_t u = dg[2 * pp] | (dg[2 * pp + 1] << 16) | kMagic2;
+              w[pp] = PREC == 0 ? ptx::sub_f16x2(u, kMagic2) : ptx::sub_bf16x2(u, kMagic2);
+            } else {
+              w[pp] = (uint32_t)__bfloat16_as_ushort(__uint2bfloat16_rn(dg[2 * pp])) |
+                      ((uint32_t)__bfloat16_as_ushort(__uint2bfloat16_rn(dg[2 * pp + 1])) << 16);
+            }
+          }
+#pragma unroll
+          for (int kg = 0; kg < 4; ++kg)
+            ptx::st_shared_v4(xs + kg * kLboR128 + r * 16, w[kg * 4 + 0], w[kg * 4 + 1],
+                              w[kg * 4 + 2], w[kg * 4 + 3]);
+        }
       }
       ptx::fence_proxy_async_smem();
       ptx::named_bar_sync(1, 64);
@@ -615,10 +662,9 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
     const bool do_last = kEpiGroups == 1 || gy == 1;  // converts the last layer
     const uint32_t hready_leader0 = ptx::mapa(bar(B_HREADY), 0);
     const uint32_t tempty_leader0 = ptx::mapa(bar(B_TEMPTY), 0);
-    const uint32_t hrow = sbase + L.h + row * 16;
     const bool own0 = kEpiGroups == 2 && gy == 0;  // group 0's private output-layer copy
     float *prm = reinterpret_cast<float *>(smem + (own0 ? L.prm0 : L.prm));  // last b | W_out | b_out
-    uint32_t *prm2 = reinterpret_cast<uint32_t *>(smem + L.prm + kPrmFloats * 4);
+    float *hbias = reinterpret_cast<float *>(smem + L.prm + kPrmFloats * 4);  // H-layer biases
     float *red = reinterpret_cast<float *>(smem + (own0 ? L.red0 : L.red));
     const uint32_t red_bar = (own0 ? 8 : 4) + q;  // named barrier of this quadrant's reduction
     const DevModel *cur = nullptr;
@@ -627,22 +673,17 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
     TileInfo nxt;
     if (t_begin < t_end) nxt = tile_info<PREC>(ts, t_begin);
     for (int64_t t = t_begin; t < t_end; ++t, ++it) {
-#ifdef LAKE_NO_PREFETCH
-      const TileInfo ti = tile_info<PREC>(ts, t);
-#else
       const TileInfo ti = nxt;
       if (t + 1 < t_end) nxt = tile_info<PREC>(ts, t + 1);
-#endif
       const int nh = ti.nh;
       if (ti.model != cur) {
-        // stage this model's epilogue parameters (each group the ones it uses): packed
-        // operand-type bias pairs of the H layers, fp32 last-layer bias | W_out | b_out
+        // stage this model's epilogue parameters (each group the ones it uses): fp32 biases
+        // of the H layers, fp32 last-layer bias | W_out | b_out
         ptx::named_bar_sync(2 + gy, NG);
         if (do_h) {
-          for (uint32_t i = et; i < (uint32_t)(nh - 1) * kHidden / 2; i += NG) {
-            const float2 bf = __ldg(reinterpret_cast<const float2 *>(ti.model->b[0]) + i);
-            prm2[i] = PREC == 0 ? ptx::pack_f16(bf.x, bf.y) : ptx::pack_bf16(bf.x, bf.y);
-          }
+          for (uint32_t i = et; i < (uint32_t)(nh - 1) * kHidden / 4; i += NG)
+            reinterpret_cast<float4 *>(hbias)[i] =
+                __ldg(reinterpret_cast<const float4 *>(ti.model->b[0]) + i);
         }
         if (do_last || (kEpiGroups == 2 && nh == 1)) {
           const float4 *src = reinterpret_cast<const float4 *>(ti.model->b[nh - 1]);
@@ -668,23 +709,12 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         LAKE_TEV(T_DFULL, it, l, warp);
         ptx::tc_fence_after();
         const uint32_t tbase = tmem + ((q * 32) << 16) + b * 256;
-        // j-th (chunk, first column) handled by this warp
-        auto chunk_of = [&](uint32_t j) { return kInterleave ? j * kEpiPerQ + hh : j; };
-        auto col_of = [&](uint32_t j) {
-          return kInterleave ? chunk_of(j) * kChunkCols : j * kChunkCols + hh * W;
-        };
+        // j-th chunk's first column handled by this warp
+        auto col_of = [&](uint32_t j) { return j * kChunkCols + hh * W; };
         const float *bl = prm;  // last-layer bias
-#ifdef LAKE_NO_EPI_PREFETCH
-        constexpr bool kPrefetch = false;
-#else
         constexpr bool kPrefetch = W <= 32;  // two W-register buffers
-#endif
         uint32_t ra[W], rb[W];  // rb unused (eliminated) without prefetch
-#ifdef LAKE_H_TMEM
-#define EPI_H(R) epi_to_h_tmem<PREC, W>(R, prm2 + l * kHidden / 2, col0, tbase)
-#else
-#define EPI_H(R) epi_to_h<PREC, W>(R, prm2 + l * kHidden / 2, col0, hrow)
-#endif
+#define EPI_H(R) epi_to_h_tmem<PREC, W>(R, hbias + l * kHidden, col0, tbase)
         ptx::tmem_ld_cols<W>(tbase + col_of(0), ra);
         ptx::tmem_ld_wait();
         if (!last) {
@@ -692,7 +722,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           // warp's next chunk is in flight while the current one is converted and stored
 #pragma unroll
           for (uint32_t j = 0; j < kWarpChunks; ++j) {
-            const uint32_t kc = chunk_of(j), col0 = col_of(j);
+            const uint32_t kc = j, col0 = col_of(j);
             if constexpr (kPrefetch) {
               if (j + 1 < kWarpChunks) {
                 if (j & 1) ptx::tmem_ld_cols<W>(tbase + col_of(j + 1), ra);
@@ -708,19 +738,11 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
               EPI_H(ra);
             }
             LAKE_TEV(T_STS, it, l, kc);
-#ifdef LAKE_H_TMEM
             ptx::tmem_st_wait();
             ptx::tc_fence_before();
-#else
-            ptx::fence_proxy_async_smem();
-#endif
             LAKE_TEV(T_FENCE, it, l, kc);
             __syncwarp();
-#ifdef LAKE_ABL_LOCALREADY
-            if (lane == 0 && rank == 0) ptx::mbar_arrive_cluster(hready_leader0 + kc * 8);
-#else
             if (lane == 0) ptx::mbar_arrive_cluster(hready_leader0 + kc * 8);
-#endif
             LAKE_TEV(T_CHUNK, it, l, kc);
             if (kPrefetch && j + 1 < kWarpChunks) ptx::tmem_ld_wait();
             LAKE_TEV(T_LDWAIT, it, l, kc);
@@ -747,6 +769,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
               epi_to_logits<W>(ra, bl, wo, col0, p);
             }
           }
+#undef EPI_H
           float p0 = p[0] + p[2], p1 = p[1] + p[3];
           // combine the kEpiPerQ warps of this quadrant (slices hh = 1.. write partials)
           if (hh > 0) {
@@ -801,24 +824,32 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
 template <int PREC, int IN_KIND>
 cudaError_t launch_t(const void *in, const TileSched &ts, int nh_layout, uint8_t *dec,
                      float *logits, cudaStream_t s, int grid) {
-  const Layout L = tc_layout(nh_layout);
-  static bool attr_set[64] = {};
+  const Layout L = tc_layout(nh_layout, PREC);
+  // per-device "attribute set" flags; a race only repeats the (idempotent) attribute call
+  static std::atomic<bool> attr_set[64];
   int dev = 0;
   cudaGetDevice(&dev);
-  if (!attr_set[dev & 63]) {
+  if (!attr_set[dev & 63].load(std::memory_order_acquire)) {
     cudaError_t e = cudaFuncSetAttribute(mlp_tc_kernel<PREC, IN_KIND>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)tc_layout(kMaxHiddenLayers).total);
+                                         (int)tc_layout(kMaxHiddenLayers, PREC).total);
     if (e != cudaSuccess) return e;
-    attr_set[dev & 63] = true;
+    attr_set[dev & 63].store(true, std::memory_order_release);
   }
   mlp_tc_kernel<PREC, IN_KIND><<<grid, kThreads, L.total, s>>>(in, ts, nh_layout, dec, logits);
   return cudaGetLastError();
 }
 
+template <int PREC>
+cudaError_t launch_p(const void *in, int in_kind, const TileSched &ts, int nh, uint8_t *dec,
+                     float *logits, cudaStream_t s, int grid) {
+  return in_kind == LAKE_IN_RAW ? launch_t<PREC, LAKE_IN_RAW>(in, ts, nh, dec, logits, s, grid)
+                                : launch_t<PREC, LAKE_IN_DIGITS>(in, ts, nh, dec, logits, s, grid);
+}
+
 }  // namespace
 
-size_t tc_smem_bytes(int nh_layout) { return tc_layout(nh_layout).total; }
+size_t tc_smem_bytes(int nh_layout, int prec) { return tc_layout(nh_layout, prec).total; }
 
 #ifdef LAKE_TRACE
 extern "C" int lake_trace_set(void *dev_buf) {
@@ -828,23 +859,21 @@ extern "C" int lake_trace_set(void *dev_buf) {
 
 cudaError_t launch_mlp_tc(const void *in, int in_kind, int prec, const TileSched &ts, int nh,
                           uint8_t *decisions, float *logits, cudaStream_t s, int device) {
-  static int sms_cache[64] = {};
-  int sms = sms_cache[device & 63];
+  static std::atomic<int> sms_cache[64];
+  int sms = sms_cache[device & 63].load(std::memory_order_relaxed);
   if (!sms) {
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
-    sms_cache[device & 63] = sms;
+    cudaError_t e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+    if (e != cudaSuccess) return e;
+    sms_cache[device & 63].store(sms, std::memory_order_relaxed);
   }
   const int64_t max_clusters = sms / 2;
   const int64_t clusters = ts.n_tiles < max_clusters ? ts.n_tiles : max_clusters;
   if (clusters <= 0) return cudaSuccess;
   const int grid = (int)(clusters * 2);
   cudaError_t e;
-  if (prec == 0)
-    e = in_kind == LAKE_IN_RAW ? launch_t<0, LAKE_IN_RAW>(in, ts, nh, decisions, logits, s, grid)
-                               : launch_t<0, LAKE_IN_DIGITS>(in, ts, nh, decisions, logits, s, grid);
-  else
-    e = in_kind == LAKE_IN_RAW ? launch_t<1, LAKE_IN_RAW>(in, ts, nh, decisions, logits, s, grid)
-                               : launch_t<1, LAKE_IN_DIGITS>(in, ts, nh, decisions, logits, s, grid);
+  if (prec == 0) e = launch_p<0>(in, in_kind, ts, nh, decisions, logits, s, grid);
+  else if (prec == 1) e = launch_p<1>(in, in_kind, ts, nh, decisions, logits, s, grid);
+  else e = launch_p<2>(in, in_kind, ts, nh, decisions, logits, s, grid);
   count_launch();
   return e;
 }

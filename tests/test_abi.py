@@ -63,8 +63,10 @@ def test_host_validation_without_device():
     # n < 0, bad flags, NULL pointers -> LAKE_ERR_INVAL before any CUDA call
     assert L.lake_linnos_infer(None, 0, -1, 0, None, None, None) == lake.LAKE_ERR_INVAL
     assert L.lake_linnos_infer(None, 0x8, 10, 0, None, None, None) == lake.LAKE_ERR_INVAL
+    # tf32 is a valid precision now: a NULL input is the argument error
     assert L.lake_linnos_infer(None, lake.LAKE_PREC_TF32, 10, 0, None, None, None) == \
-        lake.LAKE_ERR_UNSUPPORTED
+        lake.LAKE_ERR_INVAL
+    assert L.lake_linnos_infer(None, 0x50, 10, 0, None, None, None) == lake.LAKE_ERR_INVAL
     assert L.lake_linnos_infer(None, 0, 10, 0, None, None, None) == lake.LAKE_ERR_INVAL
     assert L.lake_linnos_infer(None, 0, 0, 0, None, None, None) == lake.LAKE_OK  # n == 0
     assert L.lake_linnos_digitize(None, -3, None, None) == lake.LAKE_ERR_INVAL

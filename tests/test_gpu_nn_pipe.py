@@ -30,10 +30,11 @@ def _check(lg, dec, rlg, rdec):
     assert met["agreement"] >= 0.999, met
 
 
+@pytest.mark.parametrize("prec", [lake.LAKE_PREC_F16, lake.LAKE_PREC_TF32])
 @pytest.mark.parametrize("n", [1, 255, 257, 300_001])
-def test_single_model_many_tiles(n):
+def test_single_model_many_tiles(n, prec):
     raw = inputs.device_trace("azure", n, 91, rerate=3.0)["raw"]
-    lg, dec = run_infer(400, raw, lake.LAKE_IN_RAW | lake.LAKE_PREC_F16)
+    lg, dec = run_infer(400, raw, lake.LAKE_IN_RAW | prec)
     smp = np.unique(np.concatenate([np.arange(0, n, 37), np.arange(max(0, n - 300), n)]))
     rlg, rdec = oracle.infer_raw(0, inputs.weights(0, 400), raw[smp], nthreads=0)
     _check(lg[smp], dec[smp], rlg, rdec)
@@ -43,11 +44,11 @@ def test_single_model_many_tiles(n):
     x = torch.from_numpy(raw.view(np.int32)).cuda()
     lake.digitize(x, n, d)
     torch.cuda.synchronize()
-    lg2, dec2 = run_infer(400, d.cpu().numpy(), lake.LAKE_IN_DIGITS | lake.LAKE_PREC_F16)
+    lg2, dec2 = run_infer(400, d.cpu().numpy(), lake.LAKE_IN_DIGITS | prec)
     assert np.array_equal(dec2, dec) and np.array_equal(lg2.view(np.uint32), lg.view(np.uint32))
 
 
-@pytest.mark.parametrize("prec", [lake.LAKE_PREC_F16, lake.LAKE_PREC_BF16])
+@pytest.mark.parametrize("prec", [lake.LAKE_PREC_F16, lake.LAKE_PREC_BF16, lake.LAKE_PREC_TF32])
 def test_multi_nn_equals_per_model(prec):
     raw, mids = inputs.multi_device_trace(400_000, 3, seed_base=4100, rerate=3.0)
     ids = np.array(IDS)[mids].astype(np.int32)
@@ -62,7 +63,7 @@ def test_multi_nn_equals_per_model(prec):
     assert np.all(dec[ids == 5] == 0)
 
 
-@pytest.mark.parametrize("prec", [lake.LAKE_PREC_F16, lake.LAKE_PREC_FP32])
+@pytest.mark.parametrize("prec", [lake.LAKE_PREC_F16, lake.LAKE_PREC_TF32, lake.LAKE_PREC_FP32])
 def test_many_tiny_model_groups(prec):
     """250 NN+2 models with a skewed I/O count (many groups of 1-3 I/Os): almost every tile
     of every CTA pair switches model (weight-reload protocol at its densest), plus unknown
