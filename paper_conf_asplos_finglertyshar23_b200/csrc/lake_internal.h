@@ -92,6 +92,9 @@ cudaError_t launch_mlp_fp32(const void *in, int in_kind, const TileSched &ts,
                             uint8_t *decisions, float *logits, cudaStream_t s, int device);
 cudaError_t launch_mlp_tc(const void *in, int in_kind, int prec, const TileSched &ts, int nh,
                           uint8_t *decisions, float *logits, cudaStream_t s, int device);
+// two tiles in flight per CTA pair (mlp_tc2.cu): fp16 / bf16 (prec 0 / 1)
+cudaError_t launch_mlp_tc2(const void *in, int in_kind, int prec, const TileSched &ts, int nh,
+                           int grid, uint8_t *decisions, float *logits, cudaStream_t s);
 // Grouping for infer_multi (group.cu).
 size_t group_workspace_bytes(int64_t n);
 int64_t group_max_tiles(int64_t n, int tile_rows);

@@ -38,6 +38,7 @@
 #include <cuda_fp16.h>
 
 #include <atomic>
+#include <cstdlib>
 
 #include "digitize.cuh"
 #include "lake_internal.h"
@@ -63,7 +64,8 @@ __device__ unsigned long long *g_lake_trace = nullptr;
 #endif
 enum TraceKind { T_XFULL = 1, T_TEMPTY = 2, T_HREADY = 3, T_COMMIT = 4, T_DFULL = 5,
                  T_CHUNK = 6, T_LAYER_END = 7, T_XEMPTY = 8, T_XARRIVE = 9, T_ISSUED = 10,
-                 T_LDWAIT = 11, T_STS = 12, T_FENCE = 13 };
+                 T_LDWAIT = 11, T_STS = 12, T_FENCE = 13, T_TOP = 14, T_SCHED = 15,
+                 T_WREADY = 16, T_MMA0 = 17, T_CX = 18 };
 
 // H (the next layer's A operand) stays in tensor memory, packed in place into the
 // accumulator it came from (default); -DLAKE_H_SMEM restores the SMEM H tile + proxy fences.
@@ -418,8 +420,14 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         }
       }
     }
-    // ================= MMA issuer (leader CTA, one thread) =================
-    if (rank == 0 && lane == 0) {
+    // ================= MMA issuer (leader CTA) =================
+    // The whole warp runs the schedule in converged, warp-uniform code (operands in uniform
+    // registers); only the tcgen05.mma / commit issue is predicated on lane 0. A lane-0-only
+    // region made the compiler wrap every MMA in an R2UR.BROADCAST waterfall loop whose
+    // latency, not the tensor pipe, set the issue rate (ncu: fixed-latency stalls there).
+    if (rank == 0) {
+      const bool issuer = lane == 0;
+      const uint32_t tm = __shfl_sync(0xffffffffu, tmem, 0);  // provably warp-uniform
 #ifdef LAKE_ABL_HALFN  // timing-only ablation: hidden-layer MMAs with N = 128 (half the work)
       const uint32_t idesc = ptx::umma_idesc_f16(PREC, 256, 128);
 #else
@@ -456,6 +464,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       auto slot_of = [&](int64_t tt) -> int32_t { return ts.tile_model ? ts.tile_model[tt] : -1; };
       int32_t slot_n = (t_begin + 1 < t_end) ? slot_of(t_begin + 1) : -1;
       for (int64_t t = t_begin; t < t_end; ++t, ++it) {
+        LAKE_TEV(T_TOP, it, 0, 0);
         const TileInfo ti = nxt;
         const int32_t slot_nn = (t + 2 < t_end) ? slot_of(t + 2) : -1;
         if (t + 1 < t_end) {
@@ -465,11 +474,13 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           nxt.nh = mm->nh;
         }
         slot_n = slot_nn;
+        LAKE_TEV(T_SCHED, it, 0, 0);
         if (ti.img != cur) {
           ptx::mbar_wait(bar(B_WREADY), w_phase);
           w_phase ^= 1;
           cur = ti.img;
         }
+        LAKE_TEV(T_WREADY, it, 0, 0);
         const int nh = ti.nh;
         const bool stream = streams_w2(nh, PREC);
         const uint32_t xb = (uint32_t)(it & 1);
@@ -480,16 +491,21 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           ptx::mbar_wait(bar(B_XFULL + xb), (uint32_t)((it >> 1) & 1));
           LAKE_TEV(T_XFULL, it, 0, 0);
           ptx::tc_fence_after();
-          const uint32_t d = tmem + b * 256;
+          const uint32_t d = tm + b * 256;
           const uint64_t xd = xb ? xdesc1 : xdesc0;
 #pragma unroll
-          for (uint32_t s = 0; s < kK0S; ++s)
-            ptx::mma_cg2<PREC>(d, xd + s * kStep, w0desc + s * kStep, idesc, s);
-          ptx::mma_commit_cg2(bar(B_XEMPTY + xb), 0x3);
+          for (uint32_t s = 0; s < kK0S; ++s) {
+            if (issuer) ptx::mma_cg2<PREC>(d, xd + s * kStep, w0desc + s * kStep, idesc, s);
+            LAKE_TEV(T_MMA0, it, 0, s);
+          }
+          if (issuer) ptx::mma_commit_cg2(bar(B_XEMPTY + xb), 0x3);
+          LAKE_TEV(T_CX, it, 0, 0);
           // NN: the accumulator's buffer picks the draining group (b0 -> group 0, b1 -> 1),
           // so both groups convert logits and two NN tiles are drained at once
-          ptx::mma_commit_cg2(bar((kEpiGroups == 2 && nh == 1 && b == 1 ? B_DFULLX : B_DFULL) + b),
-                              0x3);
+          if (issuer)
+            ptx::mma_commit_cg2(bar((kEpiGroups == 2 && nh == 1 && b == 1 ? B_DFULLX : B_DFULL) + b),
+                                0x3);
+          __syncwarp();
           LAKE_TEV(T_COMMIT, it, 0, 0);
           ++g;
         }
@@ -498,9 +514,9 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           acquire_buf(b);
           LAKE_TEV(T_TEMPTY, it, l, 0);
           ptx::tc_fence_after();
-          const uint32_t d = tmem + b * 256;
+          const uint32_t d = tm + b * 256;
           // A = H(l-1), in place in the previous layer's accumulator buffer
-          const uint32_t ha = tmem + ((g - 1) & 1) * 256;
+          const uint32_t ha = tm + ((g - 1) & 1) * 256;
           const bool from_ring = stream && l == 2;
           const uint64_t wd = l == 1 ? whdesc[1] : whdesc[2];
           for (uint32_t kc = 0; kc < kChunks; ++kc) {
@@ -519,11 +535,12 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
                   ptx::mbar_wait(bar(B_RFULL + slot), (mc / kTcRingSlots) & 1);
                   ptx::tc_fence_after();
                 }
-                ptx::mma_cg2_ts<PREC>(d, ha + tmem_a_col<PREC>(ks),
+                if (issuer)
+                  ptx::mma_cg2_ts<PREC>(d, ha + tmem_a_col<PREC>(ks),
                                       ringdesc + (slot * kTcRingSlotBytes >> 4) + (s % kSPS) * kStep,
                                       idesc, ks);
                 if (s % kSPS == kSPS - 1) {
-                  ptx::mma_commit_cg2(bar(B_REMPTY + slot), 0x3);
+                  if (issuer) ptx::mma_commit_cg2(bar(B_REMPTY + slot), 0x3);
                   ++mc;
                 }
               }
@@ -531,17 +548,22 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
 #pragma unroll
               for (uint32_t s = 0; s < kKS; ++s) {
                 const uint32_t ks = kc * kKS + s;
-                ptx::mma_cg2_ts<PREC>(d, ha + tmem_a_col<PREC>(ks), wd + ks * kStep, idesc, ks);
+                if (issuer)
+                  ptx::mma_cg2_ts<PREC>(d, ha + tmem_a_col<PREC>(ks), wd + ks * kStep, idesc, ks);
               }
             }
+            __syncwarp();
             LAKE_TEV(T_ISSUED, it, l, kc);
           }
-          ptx::mma_commit_cg2(bar((kEpiGroups == 2 && l + 1 == nh ? B_DFULLX : B_DFULL) + b), 0x3);
+          if (issuer)
+            ptx::mma_commit_cg2(bar((kEpiGroups == 2 && l + 1 == nh ? B_DFULLX : B_DFULL) + b), 0x3);
+          __syncwarp();
           LAKE_TEV(T_COMMIT, it, l, 0);
           ++g;
         }
-        if (t + 1 < t_end && nxt.img != cur)
+        if (t + 1 < t_end && nxt.img != cur && issuer)
           ptx::mma_commit_cg2(bar(B_WFREE), 0x3);  // old weights no longer read
+        __syncwarp();
       }
     }
   } else if (warp >= kWarpDig && warp < kWarpDig + 2) {
@@ -870,8 +892,16 @@ cudaError_t launch_mlp_tc(const void *in, int in_kind, int prec, const TileSched
   const int64_t clusters = ts.n_tiles < max_clusters ? ts.n_tiles : max_clusters;
   if (clusters <= 0) return cudaSuccess;
   const int grid = (int)(clusters * 2);
+  // Every precision runs this file's kernel. LAKE_TC_TWO_TILE=1 selects the experimental
+  // two-tiles-in-flight kernel (mlp_tc2.cu, fp16/bf16) for A/B measurements: parity-green
+  // but slower so far.
+  static const bool two_tile = [] {
+    const char *e = getenv("LAKE_TC_TWO_TILE");
+    return e && e[0] == '1';
+  }();
   cudaError_t e;
-  if (prec == 0) e = launch_p<0>(in, in_kind, ts, nh, decisions, logits, s, grid);
+  if (prec < 2 && two_tile) e = launch_mlp_tc2(in, in_kind, prec, ts, nh, grid, decisions, logits, s);
+  else if (prec == 0) e = launch_p<0>(in, in_kind, ts, nh, decisions, logits, s, grid);
   else if (prec == 1) e = launch_p<1>(in, in_kind, ts, nh, decisions, logits, s, grid);
   else e = launch_p<2>(in, in_kind, ts, nh, decisions, logits, s, grid);
   count_launch();

@@ -9,6 +9,7 @@ seeded generators); no value here comes from the CUDA path.
     m        = median(margin)
     bout'    = float32(bout[0] + m/2), float32(bout[1] - m/2)
 
+Calibration covers every model_id in [0, LAKE_MAX_MODELS), so a test may use any id.
 Calibration trace per model: device profile PROFILE_ORDER[model % 3], rerate x3,
 4096 I/Os, seed 555000 + model.
 """
@@ -24,7 +25,7 @@ sys.path.insert(0, ROOT)
 import oracle  # noqa: E402
 from paper_conf_asplos_finglertyshar23_b200.inputs import gen  # noqa: E402
 
-N_MODELS = 64
+N_MODELS = 1024  # every model_id slot (LAKE_MAX_MODELS): tests may load any id
 N_CAL = 4096
 
 

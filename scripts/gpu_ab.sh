@@ -1,12 +1,11 @@
 #!/bin/bash
-# A/B the kernel variants under build/var/*: quick parity subset + C5 bench for each
+# A/B timing of library variants (make variant VAR=name DEFS=...): C5 bench per variant
+# usage: bash scripts/gpu_ab.sh var1 var2 ...   ("base" = the product build)
 mkdir -p gpurun_out
-out=gpurun_out/ab_${1:-x}.txt
-: > $out
-for v in build/var/*/; do
-  name=$(basename $v)
-  export LAKE_LINNOS_LIB=$v/liblake_linnos.so
-  t=$(timeout 200 python -m pytest tests -m gpu -q -x -p no:cacheprovider -k "many_tiles or (tc_f16 and 20000)" 2>&1 | tail -1)
-  b=$(timeout 200 python bench.py --steps 10 --warmup 3 --no-cpu --no-e2e 2>/dev/null | python -c "import json,sys; d=json.loads(sys.stdin.read()); r=d['roofline']; print(f\"{d['value']/1e9:.3f} Ginf/s kernel {r['kernel_ms']:.3f} ms frac {r['frac']:.4f}\")")
-  echo "$name | $t | $b" >> $out
+for v in "$@"; do
+  lib=paper_conf_asplos_finglertyshar23_b200/liblake_linnos.so
+  [ "$v" != "base" ] && lib=build/var/$v/liblake_linnos.so
+  LAKE_LINNOS_LIB=$lib timeout 120 python bench.py --steps 10 --warmup 3 --no-cpu --no-e2e \
+    > gpurun_out/ab_$v.json 2> gpurun_out/ab_$v.err
+  python -c "import json;d=json.loads(open('gpurun_out/ab_$v.json').read().splitlines()[0]);print('$v', d['roofline']['kernel_ms'], d['ms_per_step'])" >> gpurun_out/ab_summary.txt 2>&1
 done
