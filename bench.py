@@ -57,6 +57,8 @@ def parse():
     p.add_argument("--sweep-out", default=None)
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu", action="store_true")
+    p.add_argument("--no-latency", action="store_true",
+                   help="skip the compact latency-vs-batch block of the default line")
     p.add_argument("--cpu-seconds", type=float, default=12.0)
     p.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                    help="control-plane backend (gloo: lets a 1-GPU box run several ranks)")
@@ -175,8 +177,8 @@ def workload(args, world, rank):
         b, e = shard.range_split(n, world, rank)
         idx = np.arange(b, e)
         mine = list(range(n_models))
-    return dict(raw=np.ascontiguousarray(raw[idx]), ids=np.ascontiguousarray(ids[idx]),
-                models={m: w["models"][m] for m in mine}, n_total=n, arch=arch,
+    return dict(raw=np.ascontiguousarray(raw[idx]), ids=np.ascontiguousarray(ids[idx]), idx=idx,
+                plan_obj=p, models={m: w["models"][m] for m in mine}, n_total=n, arch=arch,
                 n_models=n_models, plan=p["kind"], imbalance=p["imbalance"],
                 full_raw=raw, full_ids=ids, all_models=w["models"])
 
@@ -219,6 +221,95 @@ def time_oracle(wl, seconds: float):
     return dict(value=idx.size / dt, unit="inferences/s", cores=cores, kind="oracle",
                 sample=(f"stride-{stride} sample of {idx.size} of the {raw.shape[0]} I/Os "
                         f"({len(models)} models), {dt:.1f} s wall on {cores} threads"))
+
+
+# ------------------------------------------------------------------ latency vs batch (compact)
+LAT_SIZES = (1, 2, 4, 8, 16, 64, 1024, 4096)
+
+
+def latency_vs_batch(lake, local: int, reps: int = 200, warm: int = 20):
+    """BASELINE's second metric in the default line: batch latency vs batch size (Fig. 8,
+    PAPER.md P:1288-1311) for NN and NN+2 on a compact grid. Per (arch, path, b): end to end
+    through the public host-buffer call lake_linnos_infer_host (pinned host records in,
+    decisions out, stream sync; host clock, median and p99 of `reps`) and device-only (CUDA
+    events around `reps` launches of lake_linnos_infer on resident inputs); the 1-thread
+    oracle for the same batch; the crossover b (reading R22: smallest b whose GPU end-to-end
+    median beats the 1-thread oracle); and the persistent FP32 server at b = 1."""
+    import torch
+    import oracle
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream()
+    raw_all = inputs.device_trace("azure", max(LAT_SIZES), 1200, 1.0)["raw"]
+    out = {"sizes": list(LAT_SIZES), "unit": "us", "archs": {}}
+    with ClockSampler(local) as clk:
+        for arch in (0, 2):
+            blob = inputs.weights(arch, 0)
+            mid = 40 + arch
+            lake.load_weights(mid, arch, blob, local)
+            rec = {}
+            cpu = []
+            for b in LAT_SIZES:
+                raw = np.ascontiguousarray(raw_all[:b])
+                oreps = max(1, min(50, int(2e4 / (b * (1 + 15 * arch)))))
+                best = float("inf")
+                for _ in range(5 if b <= 64 else 1):  # best of 5 blocks: host-noise robust
+                    t0 = time.perf_counter()
+                    for _ in range(oreps):
+                        oracle.infer_raw(arch, blob, raw, nthreads=1)
+                    best = min(best, (time.perf_counter() - t0) * 1e6 / oreps)
+                cpu.append(round(best, 2))
+            rec["cpu_1thread_us"] = cpu
+            for prec in ("fp32", "f16"):
+                flags = lake.LAKE_IN_RAW | lake.PREC_FLAGS[prec]
+                e2e, p99, devus = [], [], []
+                for b in LAT_SIZES:
+                    raw = np.ascontiguousarray(raw_all[:b])
+                    h_in = torch.from_numpy(raw.view(np.int32)).pin_memory()
+                    h_dec = torch.empty(b, dtype=torch.uint8).pin_memory()
+                    d_in = h_in.to(dev)
+                    d_dec = torch.empty(b, dtype=torch.uint8, device=dev)
+                    stb = lake.host_staging_bytes(b, flags)
+                    stg = torch.empty(stb, dtype=torch.uint8, device=dev)
+                    for _ in range(warm):
+                        lake.infer_host(h_in, flags, b, mid, None, h_dec, None, stg, stb, stream)
+                    ts = []
+                    for _ in range(reps):
+                        t0 = time.perf_counter()
+                        lake.infer_host(h_in, flags, b, mid, None, h_dec, None, stg, stb, stream)
+                        ts.append((time.perf_counter() - t0) * 1e6)
+                    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    ev0.record(stream)
+                    for _ in range(reps):
+                        lake.infer(d_in, flags, b, mid, d_dec, None, stream)
+                    ev1.record(stream)
+                    torch.cuda.synchronize()
+                    e2e.append(round(float(np.median(ts)), 2))
+                    p99.append(round(float(np.percentile(ts, 99)), 2))
+                    devus.append(round(ev0.elapsed_time(ev1) * 1e3 / reps, 2))
+                cross = next((b for b, g, c in zip(LAT_SIZES, e2e, cpu) if g < c), None)
+                rec[prec] = {"e2e_us_median": e2e, "e2e_us_p99": p99, "device_us": devus,
+                             "crossover_batch": cross}
+            sdec = np.zeros(1, np.uint8)
+            raw1 = np.ascontiguousarray(raw_all[:1])
+            with lake.Server(mid) as srv:
+                for _ in range(warm):
+                    srv.infer(raw1, 1, sdec)
+                st = []
+                for _ in range(reps):
+                    t0 = time.perf_counter()
+                    srv.infer(raw1, 1, sdec)
+                    st.append((time.perf_counter() - t0) * 1e6)
+            rec["server_fp32_b1_us_median"] = round(float(np.median(st)), 2)
+            rec["server_crossover"] = 1 if float(np.median(st)) < cpu[0] else None
+            out["archs"][ARCH_NAME[arch]] = rec
+            lake.unload(mid, local)
+    out["clocks"] = clk.summary()
+    out["paper_context"] = ("A100 through LAKE, Fig. 8: GPU profitable for batches > 8 (NN), "
+                            "> 3 (NN+1), > 2 (NN+2); PAPER.md P:1296-1311, Table 3 P:1088")
+    out["how"] = ("e2e: lake_linnos_infer_host (pinned host buffers; zero-copy for b <= 2^14) "
+                  "median of %d after %d warm-up; device: CUDA events over %d lake_linnos_infer "
+                  "launches; cpu: oracle on 1 host thread" % (reps, warm, reps))
+    return out
 
 
 # ------------------------------------------------------------------ our implementation
@@ -279,6 +370,40 @@ def run_ours(args):
     kern_avg_max = max_over_ranks(kern_avg, dist, dev)
     n_max = max_over_ranks(float(n), dist, dev)
     value = wl["n_total"] * args.steps / (ms_max / 1e3)
+
+    # ---- multi-rank parity (outside the timed region): every rank's decisions, gathered to
+    # rank 0, must equal one rank's infer_multi over the whole batch (independent I/Os, one
+    # model per block device: PAPER.md Fig. 4 caption P:906-909) -----------------------------
+    parity = None
+    if dist is not None:
+        step(0)
+        torch.cuda.synchronize()
+        gathered = [None] * world
+        dist.all_gather_object(gathered, (wl["idx"], dec[:n].cpu().numpy()))
+        if rank == 0:
+            for m, (arch, blob) in wl["all_models"].items():
+                if m not in wl["models"]:
+                    lake.load_weights(m, arch, blob, local)
+            N = wl["n_total"]
+            fx = torch.from_numpy(wl["full_raw"].view(np.int32)).to(dev)
+            fids = torch.from_numpy(wl["full_ids"]).to(dev)
+            fdec = torch.empty(N, dtype=torch.uint8, device=dev)
+            fwsb = lake.workspace_bytes(N)
+            fws = torch.empty(fwsb, dtype=torch.uint8, device=dev)
+            lake.infer_multi(fx, flags, N, fids, fdec, None, fws, fwsb, stream)
+            torch.cuda.synchronize()
+            ref = fdec.cpu().numpy()
+            seen = np.zeros(N, dtype=np.int64)
+            bad = 0
+            for ridx, rdec in gathered:
+                seen[ridx] += 1
+                bad += int((rdec != ref[ridx]).sum())
+            parity = {"checked": int((seen == 1).sum()), "decision_mismatches": bad,
+                      "covered_once": bool(np.all(seen == 1)),
+                      "reference": "single-rank lake_linnos_infer_multi of the whole batch on rank 0",
+                      "how": "per-rank decisions all-gathered after the timed region"}
+            del fx, fids, fdec, fws
+        barrier(dist)
 
     # ---- roofline of the dominant kernel (fused MLP) -------------------------------------
     peaks = {}
@@ -351,6 +476,9 @@ def run_ours(args):
     if rank == 0 and world == 1 and not args.no_cpu:
         cpu = time_oracle(wl, args.cpu_seconds)
         cpu["value"] = round(cpu["value"], 1)
+    latency = None
+    if rank == 0 and world == 1 and not args.no_latency:
+        latency = latency_vs_batch(lake, local)
 
     if rank == 0:
         line = {
@@ -361,6 +489,8 @@ def run_ours(args):
             "data": "synthetic (seeded traces shaped like PAPER.md Table 4; random-init weights)",
             "config": config_obj(args, wl, prec, world, copies),
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+            "multi_rank_parity": parity,
+            "latency": latency,
             "gpu_launches": int(launches), "clocks": clk.summary(),
             # context, not the target (BASELINE.json north_star): the paper's claim and the
             # hardware it was measured on; beside it, this run's reduction vs the oracle

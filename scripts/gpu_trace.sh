@@ -1,5 +1,6 @@
 #!/bin/bash
-# timeline traces of the tcgen05 kernels (trace build; scripts/trace_tc.py, trace_tc2.py)
+# timeline traces of the tcgen05 kernel: SMEM-log trace build (make variant VAR=tsmem
+# DEFS="-DLAKE_TRACE -DLAKE_TRACE_SMEM"), default streams and the TMEM-quadrant streams
 mkdir -p gpurun_out
-LAKE_LINNOS_LIB=build/trace/liblake_linnos_trace.so timeout 300 python scripts/trace_tc2.py C5 f16 > gpurun_out/trace2_c5.txt 2>&1
-echo "exit $?" >> gpurun_out/trace2_c5.txt
+LAKE_TRACE_CAP=512 LAKE_LINNOS_LIB=build/var/tsmem/liblake_linnos.so timeout 300 python scripts/trace_tc.py C5 f16 > gpurun_out/trace_smem.txt 2>&1
+echo "exit $?" >> gpurun_out/trace_smem.txt

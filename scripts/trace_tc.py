@@ -16,7 +16,7 @@ KIND = {1: "XFULL", 2: "TEMPTY", 3: "HREADY", 4: "COMMIT", 5: "DFULL", 6: "CHUNK
         7: "LAYEREND", 8: "XEMPTY", 9: "XARRIVE", 10: "ISSUED", 11: "LDWAIT", 12: "STS",
         13: "FENCE", 14: "TOP", 15: "SCHED", 16: "WREADY", 17: "MMA0", 18: "CX"}
 STREAM = ({0: "mma", 1: "e3r1", 2: "e3r2", 3: "e7r1"} if os.environ.get("LAKE_TRACE_PAIR") else {0: "q0w4", 1: "q1w5", 2: "q2w6", 3: "q3w3"} if os.environ.get("LAKE_TRACE_QUAD") else {0: "mma", 1: "epi4", 2: "epi11", 3: "dig"})
-CAP = 1 << 16
+CAP = int(os.environ.get("LAKE_TRACE_CAP", 1 << 16))  # 512 for the SMEM-log build (-DLAKE_TRACE_SMEM)
 
 cfg = sys.argv[1] if len(sys.argv) > 1 else "C5"
 prec = sys.argv[2] if len(sys.argv) > 2 else "f16"
@@ -52,8 +52,10 @@ tiles = max(r[3] for r in rows) + 1
 print(f"events {len(rows)}, tiles in cluster 0: {tiles}, span {clk[-1] - clk[0]} cycles, {(clk[-1] - clk[0]) / tiles:.0f} cycles/tile")
 c0 = np.array([r[0] for r in rows if (r[2] == 4 and r[4] == 0) or (r[2] == 5 and r[4] == 0 and r[1] == 0)])
 d = np.diff(np.sort(c0))
-print(f"tile period (L0 commits): median {np.median(d):.0f} p10 {np.percentile(d, 10):.0f} p90 {np.percentile(d, 90):.0f}")
-mid = tiles // 2
+if d.size:
+    print(f"tile period (L0 commits): median {np.median(d):.0f} p10 {np.percentile(d, 10):.0f} p90 {np.percentile(d, 90):.0f}")
+present = sorted(set(r[3] for r in rows))
+mid = present[len(present) // 2 - 1] if len(present) > 2 else present[0]
 sel = [r for r in rows if r[3] in (mid, mid + 1)]
 base = sel[0][0]
 for r in sel:
