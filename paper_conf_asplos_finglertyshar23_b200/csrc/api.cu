@@ -38,10 +38,6 @@ struct DeviceState {
   DevModel host[LAKE_MAX_MODELS];
   ModelBufs bufs[LAKE_MAX_MODELS];
   DevModel *table = nullptr;  // device copy
-  // cudaFree synchronises the device, which never completes while a persistent server
-  // kernel runs: replaced buffers wait here until no server is active on the device
-  std::vector<ModelBufs> graveyard;
-  int servers = 0;
 };
 
 std::mutex g_mu;
@@ -168,27 +164,12 @@ void build_tc_image(const BlobView &v, int prec, uint8_t *img /* 2 * bytes */, s
   }
 }
 
-void free_bufs(ModelBufs &b) {
-  if (b.fp32) cudaFree(b.fp32);
-  if (b.tc) cudaFree(b.tc);
+// Release replaced model buffers: now, or once no persistent server runs (cudaFree would
+// wait forever behind a resident server kernel; deferred.cu).
+void retire_bufs(ModelBufs &b, int device) {
+  release_device(b.fp32, device);
+  release_device(b.tc, device);
   b.fp32 = b.tc = nullptr;
-}
-
-// Release replaced model buffers now, or later if a persistent server is running.
-void retire_bufs(DeviceState *st, ModelBufs &b) {
-  if (!b.fp32 && !b.tc) return;
-  if (st->servers > 0) {
-    st->graveyard.push_back(b);
-    b.fp32 = b.tc = nullptr;
-  } else {
-    free_bufs(b);
-  }
-}
-
-void flush_graveyard(DeviceState *st) {
-  if (st->servers > 0) return;
-  for (auto &b : st->graveyard) free_bufs(b);
-  st->graveyard.clear();
 }
 
 int cuda_status(cudaError_t e) {
@@ -285,7 +266,13 @@ struct ProfScope {
       cudaEvent_t a, b;
       if (cudaEventCreate(&a) != cudaSuccess) return;
       if (cudaEventCreate(&b) != cudaSuccess) { cudaEventDestroy(a); return; }
-      g_prof_ev.emplace_back(a, b);
+      try {
+        g_prof_ev.emplace_back(a, b);
+      } catch (...) {  // out of host memory: this launch is simply not profiled
+        cudaEventDestroy(a);
+        cudaEventDestroy(b);
+        return;
+      }
     }
     auto &pr = g_prof_ev[g_prof_used++];
     cudaEventRecord(pr.first, s);
@@ -382,12 +369,12 @@ int lake_linnos_load_weights(int32_t model_id, int32_t arch, const float *blob, 
   ModelBufs nb;
   if (cudaMalloc(&nb.fp32, f_total * 4) != cudaSuccess) return LAKE_ERR_NOMEM;
   if (cudaMalloc(&nb.tc, tc_total) != cudaSuccess) {
-    retire_bufs(st, nb);
+    retire_bufs(nb, device);
     return LAKE_ERR_NOMEM;
   }
   if (cudaMemcpy(nb.fp32, f.get(), f_total * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
       cudaMemcpy(nb.tc, img.get(), tc_total, cudaMemcpyHostToDevice) != cudaSuccess) {
-    retire_bufs(st, nb);
+    retire_bufs(nb, device);
     return LAKE_ERR_CUDA;
   }
   DevModel m;
@@ -405,11 +392,10 @@ int lake_linnos_load_weights(int32_t model_id, int32_t arch, const float *blob, 
   // publish: device table entry, then host mirror; retire the previous buffers. (No
   // device-wide sync: in-flight work on this model is excluded by the header's contract.)
   if (cudaMemcpy(st->table + model_id, &m, sizeof(m), cudaMemcpyHostToDevice) != cudaSuccess) {
-    retire_bufs(st, nb);
+    retire_bufs(nb, device);
     return LAKE_ERR_CUDA;
   }
-  retire_bufs(st, st->bufs[model_id]);
-  flush_graveyard(st);
+  retire_bufs(st->bufs[model_id], device);
   st->bufs[model_id] = nb;
   st->host[model_id] = m;
   return LAKE_OK;
@@ -428,8 +414,7 @@ int lake_linnos_unload(int32_t model_id, int32_t device) {
   m.arch = -1;
   if (cudaMemcpy(st->table + model_id, &m, sizeof(m), cudaMemcpyHostToDevice) != cudaSuccess)
     return LAKE_ERR_CUDA;
-  retire_bufs(st, st->bufs[model_id]);
-  flush_graveyard(st);
+  retire_bufs(st->bufs[model_id], device);
   st->host[model_id] = m;
   return LAKE_OK;
 }
@@ -804,10 +789,6 @@ int lake_linnos_server_start(int32_t model_id, lake_server_t **server_out) {
   Server *s = nullptr;
   rc = server_start(m, device, &s);
   if (rc != LAKE_OK) return rc;
-  {
-    std::lock_guard<std::mutex> lk(g_mu);
-    g_dev[device]->servers++;
-  }
   *server_out = reinterpret_cast<lake_server_t *>(s);
   return LAKE_OK;
 }
@@ -822,16 +803,7 @@ int lake_linnos_server_infer(lake_server_t *server, const lake_io_raw_t *h_raw, 
 
 int lake_linnos_server_stop(lake_server_t *server) {
   if (!server) return LAKE_ERR_INVAL;
-  const int device = server_device(reinterpret_cast<Server *>(server));
-  const int rc = server_stop(reinterpret_cast<Server *>(server));
-  std::lock_guard<std::mutex> lk(g_mu);
-  DeviceState *st = g_dev[device];
-  if (st && st->servers > 0) {
-    st->servers--;
-    DeviceGuard dg(device);
-    flush_graveyard(st);
-  }
-  return rc;
+  return server_stop(reinterpret_cast<Server *>(server));
 }
 
 uint64_t lake_linnos_launch_count(void) { return g_launches.load(); }

@@ -12,6 +12,9 @@
 // Unknown ids (out of range or not loaded) go to the tail of perm; lake_linnos_multi_grouped
 // writes decision 0 / NaN logits for them. Results do not depend on the order inside a
 // model's range (every row is computed independently), so the scatter need not be stable.
+#include <atomic>
+#include <cstddef>
+
 #include "lake_internal.h"
 
 namespace lake {
@@ -34,6 +37,11 @@ struct WsHeader {
   int64_t n_unknown;
   int32_t arch_mask;
   int32_t pad;
+  // "model slot is loaded", snapshotted once per call by group_init: histogram and scatter
+  // must classify every id identically even if another thread loads / unloads a model id
+  // (not used by this call's known models) meanwhile; a divergent view would overrun a
+  // model's reserved range of perm
+  uint8_t known[LAKE_MAX_MODELS];
 };
 
 __host__ __device__ inline size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
@@ -67,11 +75,18 @@ __device__ __forceinline__ bool known(const DevModel *table, int32_t m) {
   return m >= 0 && m < LAKE_MAX_MODELS && table[m].arch >= 0;
 }
 
-// Per-block SMEM copy of "model slot is loaded" so the per-I/O test is a shared-memory byte
-// read instead of a dependent global load of the model table.
-__device__ __forceinline__ void load_known(const DevModel *table, uint8_t *known_s) {
-  for (int m = threadIdx.x; m < LAKE_MAX_MODELS; m += blockDim.x)
-    known_s[m] = table[m].arch >= 0 ? 1 : 0;
+// Per-block SMEM copy of the call's snapshot of "model slot is loaded", so the per-I/O test
+// is a shared-memory byte read instead of a dependent global load.
+__device__ __forceinline__ void load_known(const WsHeader *h, uint8_t *known_s) {
+  for (int m = threadIdx.x; m < LAKE_MAX_MODELS; m += blockDim.x) known_s[m] = h->known[m];
+}
+
+// Zero the header and snapshot the device model table (one thread per model slot).
+__global__ void __launch_bounds__(LAKE_MAX_MODELS)
+group_init(const DevModel *__restrict__ table, WsHeader *h) {
+  uint32_t *w = reinterpret_cast<uint32_t *>(h);
+  for (uint32_t i = threadIdx.x; i < offsetof(WsHeader, known) / 4; i += blockDim.x) w[i] = 0;
+  h->known[threadIdx.x] = table[threadIdx.x].arch >= 0 ? 1 : 0;
 }
 __device__ __forceinline__ int32_t bin_of(const uint8_t *known_s, int32_t m) {
   return ((unsigned)m < (unsigned)LAKE_MAX_MODELS && known_s[m]) ? m : LAKE_MAX_MODELS;
@@ -79,11 +94,11 @@ __device__ __forceinline__ int32_t bin_of(const uint8_t *known_s, int32_t m) {
 
 template <typename IdT>
 __global__ void __launch_bounds__(kGBlock)
-group_hist(const IdT *__restrict__ ids, int64_t n, const DevModel *__restrict__ table,
-           WsHeader *h, int32_t *__restrict__ chunk_counts) {
+group_hist(const IdT *__restrict__ ids, int64_t n, WsHeader *h,
+           int32_t *__restrict__ chunk_counts) {
   __shared__ int32_t cnt[LAKE_MAX_MODELS + 1];
   __shared__ uint8_t known_s[LAKE_MAX_MODELS];
-  load_known(table, known_s);
+  load_known(h, known_s);
   for (int64_t base = (int64_t)blockIdx.x * kChunk; base < n; base += (int64_t)gridDim.x * kChunk) {
     for (int i = threadIdx.x; i <= LAKE_MAX_MODELS; i += kGBlock) cnt[i] = 0;
     __syncthreads();
@@ -155,12 +170,12 @@ group_scan(WsHeader *h) {
 
 template <typename IdT>
 __global__ void __launch_bounds__(kGBlock)
-group_scatter(const IdT *__restrict__ ids, int64_t n, const DevModel *__restrict__ table,
-              WsHeader *h, int32_t *__restrict__ perm, const int32_t *__restrict__ chunk_counts) {
+group_scatter(const IdT *__restrict__ ids, int64_t n, WsHeader *h, int32_t *__restrict__ perm,
+              const int32_t *__restrict__ chunk_counts) {
   __shared__ int32_t cnt[LAKE_MAX_MODELS + 1];
   __shared__ int32_t basep[LAKE_MAX_MODELS + 1];
   __shared__ uint8_t known_s[LAKE_MAX_MODELS];
-  load_known(table, known_s);
+  load_known(h, known_s);
   for (int64_t base = (int64_t)blockIdx.x * kChunk; base < n; base += (int64_t)gridDim.x * kChunk) {
     const int32_t *cc = chunk_counts + (base / kChunk) * kBins;  // this chunk's histogram
     for (int i = threadIdx.x; i < kBins; i += kGBlock) cnt[i] = cc[i];
@@ -280,18 +295,22 @@ static GroupPtrs group_ptrs(void *ws, int64_t n) {
 cudaError_t launch_group(int64_t n, const void *model_ids, int id_kind, const DevModel *table,
                          void *ws, int /*tile_rows*/, cudaStream_t s) {
   GroupPtrs p = group_ptrs(ws, n);
-  cudaError_t e = cudaMemsetAsync(p.h, 0, sizeof(WsHeader), s);
-  if (e != cudaSuccess) return e;
-  int dev = 0, sms = 148;
+  group_init<<<1, LAKE_MAX_MODELS, 0, s>>>(table, p.h);
+  int dev = 0;
   cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  static std::atomic<int> sms_cache[64];  // per-device SM count (a race repeats the query)
+  int sms = sms_cache[dev & 63].load(std::memory_order_relaxed);
+  if (!sms) {
+    if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) sms = 148;
+    sms_cache[dev & 63].store(sms, std::memory_order_relaxed);
+  }
   const int64_t chunks = (n + kChunk - 1) / kChunk;
   const int grid = (int)(chunks < 2 * sms ? chunks : 2 * sms);
   auto hist = [&](auto *ids) {
-    if (grid > 0) group_hist<<<grid, kGBlock, 0, s>>>(ids, n, table, p.h, p.cc);
+    if (grid > 0) group_hist<<<grid, kGBlock, 0, s>>>(ids, n, p.h, p.cc);
   };
   auto scatter = [&](auto *ids) {
-    if (grid > 0) group_scatter<<<grid, kGBlock, 0, s>>>(ids, n, table, p.h, p.perm, p.cc);
+    if (grid > 0) group_scatter<<<grid, kGBlock, 0, s>>>(ids, n, p.h, p.perm, p.cc);
   };
   const int32_t *i32 = static_cast<const int32_t *>(model_ids);
   const uint16_t *u16 = static_cast<const uint16_t *>(model_ids);
@@ -303,7 +322,7 @@ cudaError_t launch_group(int64_t n, const void *model_ids, int id_kind, const De
   group_tiles<<<(unsigned)((mt + 255) / 256), 256, 0, s>>>(p.h, p.max[0], p.max[1], p.tm[0],
                                                            p.tb[0], p.tc[0], p.tm[1], p.tb[1],
                                                            p.tc[1]);
-  count_launch(grid > 0 ? 4 : 2);
+  count_launch(grid > 0 ? 5 : 3);
   return cudaGetLastError();
 }
 

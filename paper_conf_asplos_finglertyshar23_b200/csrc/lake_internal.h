@@ -128,4 +128,10 @@ int server_device(const Server *s);
 
 void count_launch(int k = 1);
 
+// deferred.cu: releases that never block behind a running persistent server
+void release_device(void *p, int device);  // cudaFree on `device`, now or when no server runs
+void release_host(void *p);                 // cudaFreeHost, now or when no server runs
+void servers_started();
+void servers_stopped();
+
 }  // namespace lake

@@ -233,6 +233,11 @@ __device__ __forceinline__ void tmem_ld_32x32b_x8(uint32_t taddr, uint32_t (&r)[
 }
 template <int W>
 __device__ __forceinline__ void tmem_ld_cols(uint32_t taddr, uint32_t (&r)[W]) {
+#ifdef LAKE_ABL_NOLD  // timing-only ablation (mlp_tc.cu): no TMEM reads in the epilogue
+#pragma unroll
+  for (int i = 0; i < W; ++i) r[i] = taddr + i;
+  return;
+#endif
   if constexpr (W == 64) tmem_ld_32x32b_x64(taddr, r);
   else if constexpr (W == 32) tmem_ld_32x32b_x32(taddr, r);
   else if constexpr (W == 16) tmem_ld_32x32b_x16(taddr, r);

@@ -24,6 +24,7 @@
 
 #include <cmath>
 #include <cstring>
+#include <atomic>
 #include <mutex>
 #include <vector>
 
@@ -424,25 +425,26 @@ template <class Body, int RPT>
 cudaError_t fam_launch(const float *x, int64_t n, const FamModel &m, int32_t *cls, float *out,
                        cudaStream_t s, int sms) {
   const size_t smem = fam_smem_bytes<Body>(m, RPT);
-  static bool attr_set[kFamMaxDevices] = {};
+  // per-device caches shared by host threads: atomics (a race only repeats a query)
+  static std::atomic<bool> attr_set[kFamMaxDevices];
   int dev = 0;
   cudaGetDevice(&dev);
   dev &= kFamMaxDevices - 1;
-  if (!attr_set[dev]) {
+  if (!attr_set[dev].load(std::memory_order_acquire)) {
     cudaError_t e = cudaFuncSetAttribute(mlp_family_kernel<Body, RPT>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, 226 * 1024);  // + static barriers
     if (e != cudaSuccess) return e;
-    attr_set[dev] = true;
+    attr_set[dev].store(true, std::memory_order_release);
   }
   // resident CTAs per SM for this SMEM size (cached: the query costs microseconds)
-  static int occ_cache[kFamMaxDevices][64] = {};
+  static std::atomic<int> occ_cache[kFamMaxDevices][64];
   const int key = (int)((smem + 4095) / 4096) & 63;
-  int per_sm = occ_cache[dev][key];
+  int per_sm = occ_cache[dev][key].load(std::memory_order_relaxed);
   if (!per_sm) {
     cudaOccupancyMaxActiveBlocksPerMultiprocessorWithFlags(&per_sm, mlp_family_kernel<Body, RPT>,
                                                            kFamThreads, key * 4096, 0);
     if (per_sm < 1) per_sm = 1;
-    occ_cache[dev][key] = per_sm;
+    occ_cache[dev][key].store(per_sm, std::memory_order_relaxed);
   }
   const int64_t rows = (int64_t)kFamThreads * RPT;
   const int64_t tiles = (n + rows - 1) / rows;
@@ -489,7 +491,7 @@ size_t lake_mlp_blob_floats(int32_t n_layers, const int32_t *widths) {
   return t;
 }
 
-int lake_mlp_load(int32_t model_id, int32_t n_layers, const int32_t *widths, int32_t act,
+static int mlp_load_impl(int32_t model_id, int32_t n_layers, const int32_t *widths, int32_t act,
                   const float *blob, size_t n_floats, int32_t device) {
   if (model_id < 0 || model_id >= LAKE_MLP_MAX_MODELS) return LAKE_ERR_INVAL;
   if (!valid_shape(n_layers, widths)) return LAKE_ERR_INVAL;
@@ -552,17 +554,27 @@ int lake_mlp_load(int32_t model_id, int32_t n_layers, const int32_t *widths, int
   if (cudaMemcpy(d, img.data(), img.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
       (!fx.empty() && cudaMemcpy(d + img.size(), fx.data(), fx.size() * 4,
                                  cudaMemcpyHostToDevice) != cudaSuccess)) {
-    cudaFree(d);
+    release_device(d, device);
     return LAKE_ERR_CUDA;
   }
   m.img_fx = fx.empty() ? nullptr : d + img.size();
   FamSlot &s = g_fam[device]->slot[model_id];
-  if (s.dimg) cudaFree(s.dimg);
+  release_device(s.dimg, device);  // deferred while a persistent server runs
   m.img = d;
   s.m = m;
   s.dimg = d;
   s.loaded = true;
   return LAKE_OK;
+}
+
+int lake_mlp_load(int32_t model_id, int32_t n_layers, const int32_t *widths, int32_t act,
+                  const float *blob, size_t n_floats, int32_t device) {
+  // the image building allocates host vectors: never let bad_alloc cross the C ABI
+  try {
+    return mlp_load_impl(model_id, n_layers, widths, act, blob, n_floats, device);
+  } catch (...) {
+    return LAKE_ERR_NOMEM;
+  }
 }
 
 int lake_mlp_unload(int32_t model_id, int32_t device) {
@@ -573,7 +585,7 @@ int lake_mlp_unload(int32_t model_id, int32_t device) {
   FamDeviceGuard dg(device);
   if (!dg.ok) return LAKE_ERR_CUDA;
   FamSlot &s = g_fam[device]->slot[model_id];
-  cudaFree(s.dimg);
+  release_device(s.dimg, device);  // deferred while a persistent server runs
   s = FamSlot();
   return LAKE_OK;
 }
@@ -678,12 +690,12 @@ int lake_mlp_infer(const float *x, int64_t n, int32_t model_id, int32_t *classes
     if (!g_fam[device] || !g_fam[device]->slot[model_id].loaded) return LAKE_ERR_NOMODEL;
     m = g_fam[device]->slot[model_id].m;
   }
-  static int sms_cache[kFamMaxDevices] = {};
-  int sms = sms_cache[device];
+  static std::atomic<int> sms_cache[kFamMaxDevices];
+  int sms = sms_cache[device].load(std::memory_order_relaxed);
   if (!sms) {
     if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess)
       return LAKE_ERR_CUDA;
-    sms_cache[device] = sms;
+    sms_cache[device].store(sms, std::memory_order_relaxed);
   }
   // width class of the register tile; two rows per thread once the batch fills the GPU
   const int maxw = m.max_np <= 16 ? 16 : m.max_np <= 32 ? 32 : 64;

@@ -20,6 +20,8 @@
 #include <cuda_pipeline.h>
 
 #include "digitize.cuh"
+#include <atomic>
+
 #include "lake_internal.h"
 
 namespace lake {
@@ -229,14 +231,14 @@ template <int IN_KIND, int RM>
 cudaError_t launch_rm(const void *in, const TileSched &ts, uint8_t *decisions, float *logits,
                       cudaStream_t s, int64_t grid) {
   const size_t smem = sizeof(F32Smem<RM>);
-  static bool attr_set[64] = {};
+  static std::atomic<bool> attr_set[64];  // shared by host threads
   int dev = 0;
   cudaGetDevice(&dev);
-  if (!attr_set[dev & 63]) {
+  if (!attr_set[dev & 63].load(std::memory_order_acquire)) {
     cudaError_t e = cudaFuncSetAttribute(mlp_fp32_kernel<IN_KIND, RM>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    attr_set[dev & 63] = true;
+    attr_set[dev & 63].store(true, std::memory_order_release);
   }
   mlp_fp32_kernel<IN_KIND, RM><<<(unsigned)grid, kF32Threads, smem, s>>>(in, ts, decisions,
                                                                        logits);
@@ -247,11 +249,11 @@ cudaError_t launch_rm(const void *in, const TileSched &ts, uint8_t *decisions, f
 
 cudaError_t launch_mlp_fp32(const void *in, int in_kind, const TileSched &ts_in,
                             uint8_t *decisions, float *logits, cudaStream_t s, int device) {
-  static int sms_cache[64] = {};
-  int sms = sms_cache[device & 63];
+  static std::atomic<int> sms_cache[64];
+  int sms = sms_cache[device & 63].load(std::memory_order_relaxed);
   if (!sms) {
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
-    sms_cache[device & 63] = sms;
+    sms_cache[device & 63].store(sms, std::memory_order_relaxed);
   }
   TileSched ts = ts_in;
   // small single-model batches: 16-row tiles (4x less work per tile on the critical path)

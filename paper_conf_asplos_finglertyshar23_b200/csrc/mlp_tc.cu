@@ -49,6 +49,28 @@
 // per-stream event logs: stream 0 MMA thread, 1 epilogue warp 4, 2 epilogue warp 11,
 // 3 digitiser; thread-local write index (no atomics), 2 u64 per event, 64K events each
 __device__ unsigned long long *g_lake_trace = nullptr;
+#ifdef LAKE_TRACE_SMEM
+// low-overhead variant: events of tiles [LAKE_TRACE_TW0, +3) go to a 32-KB SMEM log after the
+// kernel's layout (st.shared, no global traffic) and are copied to g_lake_trace at exit;
+// 512 events per stream, fp16/bf16 only (tf32 has no SMEM to spare)
+#ifndef LAKE_TRACE_TW0
+#define LAKE_TRACE_TW0 200
+#endif
+#define LAKE_TRACE_CAP 512u
+#define LAKE_TEV(kind, tile, layer, chunk)                                                   \
+  do {                                                                                    \
+    if (tr_stream >= 0 && (tile) >= LAKE_TRACE_TW0 && (tile) < LAKE_TRACE_TW0 + 3 &&       \
+        tr_i < LAKE_TRACE_CAP) {                                                          \
+      const unsigned long long k_ = ((unsigned long long)(kind) << 56) |                   \
+          ((unsigned long long)(tile) << 24) | ((unsigned long long)(layer) << 8) |        \
+          (unsigned long long)(chunk);                                                    \
+      const unsigned long long c_ = clock64();                                            \
+      asm volatile("st.shared.v2.u64 [%0], {%1, %2};" ::                                   \
+                   "r"(tr_smem + 16u * (tr_stream * LAKE_TRACE_CAP + tr_i++)), "l"(k_),      \
+                   "l"(c_) : "memory");                                                    \
+    }                                                                                     \
+  } while (0)
+#else
 #define LAKE_TRACE_CAP (1u << 16)
 #define LAKE_TEV(kind, tile, layer, chunk)                                                   \
   do {                                                                                    \
@@ -59,6 +81,7 @@ __device__ unsigned long long *g_lake_trace = nullptr;
       p_[1] = clock64();                                                                  \
     }                                                                                     \
   } while (0)
+#endif
 #else
 #define LAKE_TEV(kind, tile, layer, chunk) do {} while (0)
 #endif
@@ -307,20 +330,27 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
 #ifdef LAKE_TRACE
   unsigned long long *const tr_buf = g_lake_trace;  // read once: events cost no global load
 #ifdef LAKE_TRACE_QUAD  // streams: epilogue warps 4, 5, 6, 3 of rank 0 (TMEM quadrants 0-3)
-  const int tr_stream = !(tr_buf && cid == 0 && rank == 0) || lane != 0 ? -1
+  int tr_stream = !(tr_buf && cid == 0 && rank == 0) || lane != 0 ? -1
                       : (warp >= kWarpEpi && warp < kWarpEpi + 4) ? (int)((warp - kWarpEpi + 3) & 3) : -1;
 #elif defined(LAKE_TRACE_PAIR)  // streams: MMA, epilogue warp 3 of rank 0 / rank 1, warp 7 of rank 0
-  const int tr_stream = !(tr_buf && cid == 0) || lane != 0 ? -1
+  int tr_stream = !(tr_buf && cid == 0) || lane != 0 ? -1
                       : (warp == kWarpMma && rank == 0) ? 0
                       : (warp == kWarpEpi && rank == 0) ? 1
                       : (warp == kWarpEpi && rank == 1) ? 2
                       : (warp == kWarpEpi + 4 && rank == 0) ? 3 : -1;
 #else
-  const int tr_stream = !(tr_buf && cid == 0 && rank == 0) ? -1
+  int tr_stream = !(tr_buf && cid == 0 && rank == 0) ? -1
                       : (warp == kWarpMma && lane == 0) ? 0 : (warp == kWarpEpi && lane == 0) ? 1
                       : (warp == kWarpMma - 1 && lane == 0) ? 2 : (threadIdx.x == 0) ? 3 : -1;
 #endif
   uint32_t tr_i = 0;
+#ifdef LAKE_TRACE_SMEM
+  const uint32_t tr_smem = sbase + L.total;
+  if (tr_buf && cid == 0 && rank == 0)  // clear the log (keys 0 = unused)
+    for (uint32_t i = threadIdx.x; i < 4 * LAKE_TRACE_CAP * 4; i += blockDim.x)
+      reinterpret_cast<uint32_t *>(smem + L.total)[i] = 0;
+  if (PREC == 2) tr_stream = -1;
+#endif
 #endif
   const int64_t n_tiles = ts.n_tiles_dev ? (int64_t)*ts.n_tiles_dev : ts.n_tiles;
   const int64_t t_begin = n_tiles * cid / ncl;
@@ -520,7 +550,9 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           const bool from_ring = stream && l == 2;
           const uint64_t wd = l == 1 ? whdesc[1] : whdesc[2];
           for (uint32_t kc = 0; kc < kChunks; ++kc) {
+#ifndef LAKE_ABL_NOHREADY  // timing-only ablation: the MMA never waits for H chunks
             ptx::mbar_wait(bar(B_HREADY + kc), (h_phase >> kc) & 1);
+#endif
             h_phase ^= (1u << kc);
             LAKE_TEV(T_HREADY, it, l, kc);
             ptx::tc_fence_after();
@@ -721,12 +753,20 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         const uint32_t b = g & 1;
         const bool nn2 = kEpiGroups == 2 && nh == 1;  // NN: buffer b is drained by group b
         if (nn2 ? gy != b : !(last ? do_last : do_h)) continue;
-        if (kEpiGroups == 2 && (nn2 ? b == 1 : last)) {
-          ptx::mbar_wait(bar(B_DFULLX + b), (dx_phase >> b) & 1);
-          dx_phase ^= (1u << b);
-        } else {
-          ptx::mbar_wait(bar(B_DFULL + b), (d_phase >> b) & 1);
-          d_phase ^= (1u << b);
+        {
+          const bool x = kEpiGroups == 2 && (nn2 ? b == 1 : last);
+          const uint32_t wb = x ? bar(B_DFULLX + b) : bar(B_DFULL + b);
+          const uint32_t wp = ((x ? dx_phase : d_phase) >> b) & 1;
+#ifdef LAKE_POLL1
+          // one warp of the group polls the mbarrier, the others wait on a named barrier
+          // (no try_wait traffic from 8 warps through the SYNCS unit the MMA thread uses)
+          if (lw == 0) ptx::mbar_wait(wb, wp);
+          ptx::named_bar_sync(2 + gy, NG);
+#else
+          ptx::mbar_wait(wb, wp);
+#endif
+          if (x) dx_phase ^= (1u << b);
+          else d_phase ^= (1u << b);
         }
         LAKE_TEV(T_DFULL, it, l, warp);
         ptx::tc_fence_after();
@@ -841,6 +881,11 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
     ptx::tc_fence_after();
     ptx::tmem_dealloc_cg2(tmem, 512);
   }
+#if defined(LAKE_TRACE) && defined(LAKE_TRACE_SMEM)
+  if (PREC != 2 && tr_buf && cid == 0 && rank == 0)
+    for (uint32_t i = threadIdx.x; i < 4 * LAKE_TRACE_CAP * 2; i += blockDim.x)
+      tr_buf[i] = reinterpret_cast<const unsigned long long *>(smem + L.total)[i];
+#endif
 }
 
 template <int PREC, int IN_KIND>
@@ -854,11 +899,23 @@ cudaError_t launch_t(const void *in, const TileSched &ts, int nh_layout, uint8_t
   if (!attr_set[dev & 63].load(std::memory_order_acquire)) {
     cudaError_t e = cudaFuncSetAttribute(mlp_tc_kernel<PREC, IN_KIND>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)tc_layout(kMaxHiddenLayers, PREC).total);
+                                         (int)tc_layout(kMaxHiddenLayers, PREC).total +
+#if defined(LAKE_TRACE) && defined(LAKE_TRACE_SMEM)
+                                             (PREC == 2 ? 0 : 4 * LAKE_TRACE_CAP * 16)
+#else
+                                             0
+#endif
+                                         );
     if (e != cudaSuccess) return e;
     attr_set[dev & 63].store(true, std::memory_order_release);
   }
-  mlp_tc_kernel<PREC, IN_KIND><<<grid, kThreads, L.total, s>>>(in, ts, nh_layout, dec, logits);
+#if defined(LAKE_TRACE) && defined(LAKE_TRACE_SMEM)
+  constexpr uint32_t kTraceBytes = PREC == 2 ? 0u : 4u * LAKE_TRACE_CAP * 16u;
+#else
+  constexpr uint32_t kTraceBytes = 0;
+#endif
+  mlp_tc_kernel<PREC, IN_KIND><<<grid, kThreads, L.total + kTraceBytes, s>>>(in, ts, nh_layout, dec,
+                                                                            logits);
   return cudaGetLastError();
 }
 

@@ -278,11 +278,12 @@ int server_start(const DevModel &m, int device, Server **out) {
     e = cudaFuncSetAttribute(server_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)sizeof(ServerSmem));
   if (e != cudaSuccess) {
-    cudaFreeHost(s->host);
+    release_host(s->host);
     delete s;
     return LAKE_ERR_CUDA;
   }
   uint8_t *d = static_cast<uint8_t *>(d_host);
+  servers_started();  // from here on, library frees defer until the last server stops
   server_kernel<<<kCtas, kThreadsS, sizeof(ServerSmem), s->stream>>>(
       m, reinterpret_cast<Mailbox *>(d), reinterpret_cast<const uint32_t *>(d + sizeof(Mailbox)),
       d + sizeof(Mailbox) + LAKE_SERVER_MAX_BATCH * 36,
@@ -296,8 +297,9 @@ int server_start(const DevModel &m, int device, Server **out) {
   }
   if (e != cudaSuccess) {
     cudaStreamDestroy(s->stream);
-    cudaFreeHost(s->host);
+    release_host(s->host);
     delete s;
+    servers_stopped();
     return LAKE_ERR_CUDA;
   }
   *out = s;
@@ -330,10 +332,11 @@ int server_infer(Server *s, const lake_io_raw_t *raw, int32_t n, uint8_t *dec, f
 int server_stop(Server *s) {
   __sync_synchronize();
   s->mb->seq_in = kStop;
-  cudaError_t e = cudaStreamSynchronize(s->stream);
+  cudaError_t e = cudaStreamSynchronize(s->stream);  // this server's kernel only
   cudaStreamDestroy(s->stream);
-  cudaFreeHost(s->host);
+  release_host(s->host);  // parked while other servers still run (deferred.cu)
   delete s;
+  servers_stopped();
   return e == cudaSuccess ? LAKE_OK : LAKE_ERR_CUDA;
 }
 

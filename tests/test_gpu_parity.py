@@ -557,3 +557,46 @@ def test_server_survives_unload():
     srv.stop()
     _, rdec = oracle.infer_raw(2, inputs.weights(2, 555), raw, nthreads=0)
     assert np.array_equal(h_dec, rdec)
+
+
+_TWO_SERVERS = r"""
+import sys, numpy as np
+sys.path.insert(0, sys.argv[1])
+import torch
+import oracle
+from paper_conf_asplos_finglertyshar23_b200 import inputs, lake
+from paper_conf_asplos_finglertyshar23_b200.inputs import family
+torch.cuda.set_device(0)
+for m, a in ((560, 2), (561, 0)):
+    lake.load_weights(m, a, inputs.weights(a, m), 0)
+raw = np.ascontiguousarray(inputs.device_trace("azure", 40, 3, rerate=3.0)["raw"])
+s1, s2 = lake.Server(560), lake.Server(561)
+d = np.zeros(40, np.uint8)
+s1.infer(raw, 40, d)
+s1.stop()                                   # a second server is still resident
+cfg = family.FAMILY["mllb"]
+lake.mlp_load(3, cfg["widths"], cfg["act"], family.weights(cfg["widths"], 0), 0)
+lake.mlp_load(3, cfg["widths"], cfg["act"], family.weights(cfg["widths"], 1), 0)  # replace
+lake.mlp_unload(3, 0)
+lake.load_weights(560, 2, inputs.weights(2, 560), 0)   # replace while s2 runs
+lake.unload(560, 0)
+s2.infer(raw, 40, d)
+_, rdec = oracle.infer_raw(0, inputs.weights(0, 561), raw, nthreads=0)
+assert np.array_equal(d, rdec)
+s2.stop()
+lake.unload(561, 0)
+print("ok")
+"""
+
+
+def test_two_servers_and_frees_while_one_runs():
+    """stopping one of two servers, and replacing / unloading LinnOS and MLP-family
+    models while a server is resident, must not block (frees are deferred until the last
+    server stops); run in a subprocess under a timeout so a regression cannot hang the suite."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = subprocess.run([sys.executable, "-c", _TWO_SERVERS, root], capture_output=True,
+                         text=True, timeout=300)
+    assert out.returncode == 0 and out.stdout.strip().endswith("ok"), out.stderr[-2000:]
