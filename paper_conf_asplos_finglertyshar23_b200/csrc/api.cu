@@ -482,7 +482,10 @@ size_t lake_linnos_workspace_bytes(int64_t n) {
 }
 
 int multi_group_impl(int64_t n, const void *model_ids, int id_kind, void *workspace,
-                     size_t ws_bytes, void *stream);
+                     size_t ws_bytes, void *stream, const void *in = nullptr, int in_kind = 0);
+int multi_grouped_impl(const void *in, uint32_t flags, int64_t n, uint8_t *decisions,
+                       float *logits, void *workspace, size_t ws_bytes, void *stream,
+                       bool packed);
 
 int lake_linnos_multi_group(int64_t n, const int32_t *model_ids, void *workspace,
                             size_t ws_bytes, void *stream) {
@@ -490,7 +493,7 @@ int lake_linnos_multi_group(int64_t n, const int32_t *model_ids, void *workspace
 }
 
 int multi_group_impl(int64_t n, const void *model_ids, int id_kind, void *workspace,
-                     size_t ws_bytes, void *stream) {
+                     size_t ws_bytes, void *stream, const void *in, int in_kind) {
   if (n < 0 || n > (int64_t)INT32_MAX) return LAKE_ERR_INVAL;
   if (n > 0 && !model_ids) return LAKE_ERR_INVAL;
   if (!workspace) return LAKE_ERR_INVAL;
@@ -509,11 +512,18 @@ int multi_group_impl(int64_t n, const void *model_ids, int id_kind, void *worksp
     table = st->table;
   }
   return cuda_status(
-      launch_group(n, model_ids, id_kind, table, workspace, 0, static_cast<cudaStream_t>(stream)));
+      launch_group(n, model_ids, id_kind, table, workspace, in, in_kind,
+                   static_cast<cudaStream_t>(stream)));
 }
 
 int lake_linnos_multi_grouped(const void *in, uint32_t flags, int64_t n, uint8_t *decisions,
                               float *logits, void *workspace, size_t ws_bytes, void *stream) {
+  return multi_grouped_impl(in, flags, n, decisions, logits, workspace, ws_bytes, stream, false);
+}
+
+int multi_grouped_impl(const void *in, uint32_t flags, int64_t n, uint8_t *decisions,
+                       float *logits, void *workspace, size_t ws_bytes, void *stream,
+                       bool packed) {
   if (n < 0 || n > (int64_t)INT32_MAX) return LAKE_ERR_INVAL;
   int in_kind, prec;
   int rc = check_flags(flags, n, &in_kind, &prec);
@@ -530,6 +540,10 @@ int lake_linnos_multi_grouped(const void *in, uint32_t flags, int64_t n, uint8_t
   cudaError_t e = launch_unknown_fill(workspace, n, decisions, logits, s);
   if (e != cudaSuccess) return cuda_status(e);
   if (!table || !any) return LAKE_OK;
+  if (prec >= 0 && !packed) {  // grouped by a separate multi_group call: pack through perm
+    e = launch_group_pack(workspace, n, in, in_kind, s);
+    if (e != cudaSuccess) return cuda_status(e);
+  }
   TileSched ts;
   std::memset(&ts, 0, sizeof(ts));
   group_sched(workspace, n, prec < 0 ? 0 : 1, table, &ts);
@@ -546,10 +560,13 @@ int lake_linnos_infer_multi(const void *in, uint32_t flags, int64_t n, const int
   if (n == 0) return LAKE_OK;
   if (!in || !decisions || !model_ids || !workspace) return LAKE_ERR_INVAL;
   if (check_input_ptr(in, in_kind) != LAKE_OK) return LAKE_ERR_INVAL;
-  rc = multi_group_impl(n, model_ids, id_kind_of(flags), workspace, ws_bytes, stream);
+  // tensor-core paths: the scatter also packs every I/O's digit row in grouped order (read
+  // in arrival order, coalesced), which the fused kernel then bulk-copies per tile
+  rc = multi_group_impl(n, model_ids, id_kind_of(flags), workspace, ws_bytes, stream,
+                        prec >= 0 ? in : nullptr, in_kind);
   if (rc != LAKE_OK) return rc;
-  return lake_linnos_multi_grouped(in, flags & ~(uint32_t)LAKE_IDS_MASK, n, decisions, logits,
-                                   workspace, ws_bytes, stream);
+  return multi_grouped_impl(in, flags & ~(uint32_t)LAKE_IDS_MASK, n, decisions, logits,
+                            workspace, ws_bytes, stream, prec >= 0);
 }
 
 int lake_linnos_multi_status(const void *workspace, size_t ws_bytes, int64_t *n_unknown,

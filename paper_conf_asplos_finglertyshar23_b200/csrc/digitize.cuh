@@ -46,3 +46,40 @@ __device__ __forceinline__ void digitize_record(const uint32_t (&rec)[9], F &&f)
 }
 
 }  // namespace lake
+
+namespace lake {
+
+// Packed digit row (internal workspace format, 16 B per I/O): digit k (0..30) in the nibble
+// (k & 1) of byte k/2 (low nibble first); nibble 31 is 0. Written by the grouping pass in
+// model-grouped order so the fused tensor-core kernel can bulk-copy contiguous rows.
+__device__ __forceinline__ uint4 pack_digits(const uint32_t (&dg)[32]) {
+  uint32_t w[4];
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    uint32_t v = 0;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) v |= (dg[q * 8 + j] & 0xFu) << (4 * j);
+    w[q] = v;
+  }
+  return make_uint4(w[0], w[1], w[2], w[3]);
+}
+
+// Packed row of one raw record.
+__device__ __forceinline__ uint4 pack_record(const uint32_t (&rec)[9]) {
+  uint32_t dg[32];
+#pragma unroll
+  for (int i = 0; i < 32; ++i) dg[i] = 0;
+  digitize_record(rec, [&](int k, uint32_t v) { dg[k] = v; });
+  return pack_digits(dg);
+}
+
+// Packed row of a LAKE_IN_DIGITS row (bytes 0..30 are digits 0..9).
+__device__ __forceinline__ uint4 pack_digit_bytes(const uint4 lo, const uint4 hi) {
+  const uint32_t b[8] = {lo.x, lo.y, lo.z, lo.w, hi.x, hi.y, hi.z, hi.w};
+  uint32_t dg[32];
+#pragma unroll
+  for (int k = 0; k < 32; ++k) dg[k] = k < 31 ? (b[k >> 2] >> ((k & 3) * 8)) & 0xFFu : 0u;
+  return pack_digits(dg);
+}
+
+}  // namespace lake

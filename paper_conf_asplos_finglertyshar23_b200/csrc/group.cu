@@ -14,7 +14,9 @@
 // model's range (every row is computed independently), so the scatter need not be stable.
 #include <atomic>
 #include <cstddef>
+#include <type_traits>
 
+#include "digitize.cuh"
 #include "lake_internal.h"
 
 namespace lake {
@@ -48,7 +50,7 @@ __host__ __device__ inline size_t align256(size_t x) { return (x + 255) & ~(size
 
 struct WsLayout {
   size_t header, perm, t64_model, t64_begin, t64_count, t256_model, t256_begin, t256_count,
-      chunk_counts, total;
+      chunk_counts, pdig, total;
   int64_t max64, max256;
 };
 
@@ -67,6 +69,9 @@ WsLayout ws_layout(int64_t n) {
   L.t256_count = off; off = align256(off + (size_t)L.max256 * 4);
   // per-chunk histograms written by group_hist, read back by group_scatter (no recount)
   L.chunk_counts = off; off = align256(off + (size_t)((n + kChunk - 1) / kChunk) * kBins * 4);
+  // packed digit rows (16 B per I/O) in model-grouped order, for the tensor-core kernel's
+  // contiguous bulk-copy staging
+  L.pdig = off; off = align256(off + (size_t)n * 16);
   L.total = off;
   return L;
 }
@@ -79,6 +84,21 @@ __device__ __forceinline__ bool known(const DevModel *table, int32_t m) {
 // is a shared-memory byte read instead of a dependent global load.
 __device__ __forceinline__ void load_known(const WsHeader *h, uint8_t *known_s) {
   for (int m = threadIdx.x; m < LAKE_MAX_MODELS; m += blockDim.x) known_s[m] = h->known[m];
+}
+
+// Packed digit row of I/O i of the caller's input.
+template <int IN_KIND>
+__device__ __forceinline__ uint4 pack_input(const void *in, int64_t i) {
+  if constexpr (IN_KIND == LAKE_IN_RAW) {
+    const uint32_t *src = static_cast<const uint32_t *>(in) + i * 9;
+    uint32_t rec[9];
+#pragma unroll
+    for (int f = 0; f < 9; ++f) rec[f] = __ldg(src + f);
+    return pack_record(rec);
+  } else {
+    const uint4 *src = reinterpret_cast<const uint4 *>(static_cast<const uint8_t *>(in) + i * 32);
+    return pack_digit_bytes(__ldg(src), __ldg(src + 1));
+  }
 }
 
 // Zero the header and snapshot the device model table (one thread per model slot).
@@ -168,10 +188,13 @@ group_scan(WsHeader *h) {
   }
 }
 
-template <typename IdT>
+// in_kind < 0: perm only; LAKE_IN_RAW / LAKE_IN_DIGITS: also the packed digit row of every
+// known I/O at its grouped position (the I/O's input is read in arrival order: coalesced).
+template <typename IdT, int IN_KIND>
 __global__ void __launch_bounds__(kGBlock)
 group_scatter(const IdT *__restrict__ ids, int64_t n, WsHeader *h, int32_t *__restrict__ perm,
-              const int32_t *__restrict__ chunk_counts) {
+              const int32_t *__restrict__ chunk_counts, const void *__restrict__ in,
+              uint4 *__restrict__ pdig) {
   __shared__ int32_t cnt[LAKE_MAX_MODELS + 1];
   __shared__ int32_t basep[LAKE_MAX_MODELS + 1];
   __shared__ uint8_t known_s[LAKE_MAX_MODELS];
@@ -191,9 +214,23 @@ group_scatter(const IdT *__restrict__ ids, int64_t n, WsHeader *h, int32_t *__re
       const int32_t m = bin_of(known_s, (int32_t)__ldg(ids + i));
       const int32_t r = atomicAdd(&cnt[m], 1);
       perm[basep[m] + r] = (int32_t)i;
+      if constexpr (IN_KIND >= 0) {
+        if (m < LAKE_MAX_MODELS) pdig[basep[m] + r] = pack_input<IN_KIND>(in, i);
+      }
     }
     __syncthreads();
   }
+}
+
+// multi_grouped after a separate multi_group call: packed rows gathered through perm
+template <int IN_KIND>
+__global__ void __launch_bounds__(256)
+group_pack(const WsHeader *__restrict__ h, const int32_t *__restrict__ perm,
+           const void *__restrict__ in, uint4 *__restrict__ pdig) {
+  const int64_t nk = h->n_known;
+  for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < nk;
+       p += (int64_t)gridDim.x * blockDim.x)
+    pdig[p] = pack_input<IN_KIND>(in, perm[p]);
 }
 
 __device__ __forceinline__ int find_model(const int32_t *off, int32_t t) {
@@ -270,6 +307,7 @@ struct GroupPtrs {
   int32_t *nt[2];
   int64_t max[2];
   int32_t *cc;  // per-chunk histograms
+  uint4 *pdig;  // packed digit rows, grouped order
 };
 
 static GroupPtrs group_ptrs(void *ws, int64_t n) {
@@ -285,6 +323,7 @@ static GroupPtrs group_ptrs(void *ws, int64_t n) {
   p.tb[1] = reinterpret_cast<int64_t *>(b + L.t256_begin);
   p.tc[1] = reinterpret_cast<int32_t *>(b + L.t256_count);
   p.cc = reinterpret_cast<int32_t *>(b + L.chunk_counts);
+  p.pdig = reinterpret_cast<uint4 *>(b + L.pdig);
   p.nt[0] = &p.h->n_tiles64;
   p.nt[1] = &p.h->n_tiles256;
   p.max[0] = L.max64;
@@ -293,7 +332,7 @@ static GroupPtrs group_ptrs(void *ws, int64_t n) {
 }
 
 cudaError_t launch_group(int64_t n, const void *model_ids, int id_kind, const DevModel *table,
-                         void *ws, int /*tile_rows*/, cudaStream_t s) {
+                         void *ws, const void *in, int in_kind, cudaStream_t s) {
   GroupPtrs p = group_ptrs(ws, n);
   group_init<<<1, LAKE_MAX_MODELS, 0, s>>>(table, p.h);
   int dev = 0;
@@ -310,7 +349,14 @@ cudaError_t launch_group(int64_t n, const void *model_ids, int id_kind, const De
     if (grid > 0) group_hist<<<grid, kGBlock, 0, s>>>(ids, n, p.h, p.cc);
   };
   auto scatter = [&](auto *ids) {
-    if (grid > 0) group_scatter<<<grid, kGBlock, 0, s>>>(ids, n, p.h, p.perm, p.cc);
+    using IdT = std::remove_cv_t<std::remove_pointer_t<decltype(ids)>>;
+    if (grid <= 0) return;
+    if (!in)
+      group_scatter<IdT, -1><<<grid, kGBlock, 0, s>>>(ids, n, p.h, p.perm, p.cc, nullptr, nullptr);
+    else if (in_kind == LAKE_IN_RAW)
+      group_scatter<IdT, LAKE_IN_RAW><<<grid, kGBlock, 0, s>>>(ids, n, p.h, p.perm, p.cc, in, p.pdig);
+    else
+      group_scatter<IdT, LAKE_IN_DIGITS><<<grid, kGBlock, 0, s>>>(ids, n, p.h, p.perm, p.cc, in, p.pdig);
   };
   const int32_t *i32 = static_cast<const int32_t *>(model_ids);
   const uint16_t *u16 = static_cast<const uint16_t *>(model_ids);
@@ -327,8 +373,19 @@ cudaError_t launch_group(int64_t n, const void *model_ids, int id_kind, const De
 }
 
 // Fill a TileSched for the grouped launch; which = 0 (64-row FP32 tiles) / 1 (256-row TC).
+cudaError_t launch_group_pack(void *ws, int64_t n, const void *in, int in_kind, cudaStream_t s) {
+  GroupPtrs p = group_ptrs(ws, n);
+  const int grid = (int)((n + 255) / 256 < 4 * 148 ? (n + 255) / 256 : 4 * 148);
+  if (grid <= 0) return cudaSuccess;
+  if (in_kind == LAKE_IN_RAW) group_pack<LAKE_IN_RAW><<<grid, 256, 0, s>>>(p.h, p.perm, in, p.pdig);
+  else group_pack<LAKE_IN_DIGITS><<<grid, 256, 0, s>>>(p.h, p.perm, in, p.pdig);
+  count_launch();
+  return cudaGetLastError();
+}
+
 void group_sched(void *ws, int64_t n, int which, const DevModel *table, TileSched *ts) {
   GroupPtrs p = group_ptrs(ws, n);
+  ts->pdig = which == 1 ? p.pdig : nullptr;
   ts->tile_model = p.tm[which];
   ts->tile_begin = p.tb[which];
   ts->tile_count = p.tc[which];

@@ -78,6 +78,7 @@ struct TileSched {
   const int64_t *tile_begin;   // [n_tiles] first position in `perm`
   const int32_t *tile_count;   // [n_tiles] rows in the tile
   const int32_t *perm;         // position -> I/O index, or nullptr (identity)
+  const uint4 *pdig;           // packed digit rows in position order (multi, TC), or nullptr
   const int32_t *n_tiles_dev;  // device tile count (multi) or nullptr
   int64_t n_tiles;             // host tile count (single) / upper bound (multi)
   int64_t n;                   // I/Os
@@ -99,8 +100,11 @@ cudaError_t launch_mlp_tc2(const void *in, int in_kind, int prec, const TileSche
 size_t group_workspace_bytes(int64_t n);
 int64_t group_max_tiles(int64_t n, int tile_rows);
 // id_kind: 0 int32, 1 uint16, 2 uint8 (flags bits 8..9)
+// in != nullptr: the scatter also writes the packed digit rows of `in` (in_kind) in grouped
+// order; otherwise launch_group_pack fills them later by gathering through perm
 cudaError_t launch_group(int64_t n, const void *model_ids, int id_kind, const DevModel *table,
-                         void *ws, int tile_rows, cudaStream_t s);
+                         void *ws, const void *in, int in_kind, cudaStream_t s);
+cudaError_t launch_group_pack(void *ws, int64_t n, const void *in, int in_kind, cudaStream_t s);
 // which = 0: 64-row FP32 tiles, 1: 256-row tensor-core tiles
 void group_sched(void *ws, int64_t n, int which, const DevModel *table, TileSched *ts);
 cudaError_t launch_unknown_fill(void *ws, int64_t n, uint8_t *decisions, float *logits,

@@ -153,15 +153,19 @@ __host__ __device__ constexpr bool streams_w2(int nh, int prec) {
   return tc_resident_bytes(nh, prec) < tc_image_bytes(nh, prec);
 }
 
+// input staging (digitisers): two buffers of 128 rows; tf32 only has room for packed rows
+__host__ __device__ constexpr uint32_t kStageBytes(int prec) { return prec == 2 ? 2048u : 4608u; }
+
 struct Layout {
-  uint32_t ring, h, x, prm, red, prm0, red0, bar, total;
+  uint32_t ring, h, x, stage, prm, red, prm0, red0, bar, total;
 };
 __host__ __device__ constexpr Layout tc_layout(int nh_layout, int prec) {
   Layout L{};
   L.ring = align1k(tc_resident_bytes(nh_layout, prec));
   L.h = L.ring + (streams_w2(nh_layout, prec) ? kTcRingSlots * kTcRingSlotBytes : 0u);
   L.x = L.h + kHBytes;
-  L.prm = L.x + 2 * x_bytes(prec);
+  L.stage = L.x + 2 * x_bytes(prec);
+  L.prm = L.stage + 2 * kStageBytes(prec);
   L.red = L.prm + kPrmFloats * 4 + kPrm2Words * 4;
   // group 0's own copy of the output-layer parameters and partial sums: with two epilogue
   // groups, NN tiles (a single layer) are drained by the group of their accumulator buffer
@@ -180,7 +184,8 @@ enum : uint32_t {
   B_TEMPTY = 10, B_HREADY = 12, B_WFREE = 12 + kChunks,
   B_RFULL = 13 + kChunks,                 // [kTcRingSlots] W2 ring slot loaded (tf32 NN+2)
   B_REMPTY = B_RFULL + kTcRingSlots,      // [kTcRingSlots] W2 ring slot consumed
-  B_COUNT = B_REMPTY + kTcRingSlots
+  B_SFULL = B_REMPTY + kTcRingSlots,     // [2] input staging buffer loaded (bulk copy)
+  B_COUNT = B_SFULL + 2
 };
 constexpr uint32_t kTmemSlot = B_COUNT * 8;  // u32 TMEM base address
 static_assert(kTmemSlot + 4 <= 256, "barrier block");
@@ -374,6 +379,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       ptx::mbar_init(bar(B_RFULL + i), rank == 0 ? 2 : 1);
       ptx::mbar_init(bar(B_REMPTY + i), 1);      // tcgen05.commit (multicast)
     }
+    for (int i = 0; i < 2; ++i) ptx::mbar_init(bar(B_SFULL + i), 1);  // expect_tx arrive
     ptx::fence_mbar_init();
   }
   if (warp == kWarpLoad) {
@@ -599,75 +605,160 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       }
     }
   } else if (warp >= kWarpDig && warp < kWarpDig + 2) {
-    // ================= digitisers: raw -> X (operand-type digits), 2 rows per thread ======
-    // Both rows' gathers are issued before any shared store (the st.shared asm carries a
-    // memory clobber, so loads written after it could not be hoisted): the two rows' global
-    // latencies overlap.
+    // ================= digitisers: input rows -> X (operand-type digits) ===============
+    // Each CTA's 128 rows of a tile are contiguous in one of three staged formats, brought
+    // into SMEM by a bulk copy (cp.async.bulk, TMA engine) two tiles ahead and converted from
+    // there (2 rows per thread):
+    //   packed  multi-model calls: the grouping pass wrote every I/O's packed digit row
+    //           (16 B, digitize.cuh) in model-grouped order -> ts.pdig
+    //   raw     single-model calls, LAKE_IN_RAW, 16-B aligned input: 36-B records
+    //   digits  single-model calls, LAKE_IN_DIGITS, 16-B aligned input: 32-B rows
+    // Anything else (misaligned input, or rows too large for this precision's staging
+    // buffers) gathers each row with global loads (the fallback below).
     const uint32_t d = threadIdx.x - kWarpDig * 32;  // 0..63
     const uint32_t xfull_leader0 = ptx::mapa(bar(B_XFULL), 0);
+    const uint32_t row_bytes = ts.pdig ? 16u : (IN_KIND == LAKE_IN_RAW ? 36u : 32u);
+#ifdef LAKE_ABL_NOSTAGE  // A/B switch: always the gather path
+    const bool staged = false;
+#else
+    const bool staged = ts.pdig != nullptr ||
+                        (ts.perm == nullptr && (reinterpret_cast<uintptr_t>(in) & 15) == 0 &&
+                         128u * row_bytes <= kStageBytes(PREC));
+#endif
+    const uint8_t *stage_src = ts.pdig ? reinterpret_cast<const uint8_t *>(ts.pdig)
+                                       : static_cast<const uint8_t *>(in);
+    // rows of tile t in this CTA, and the 16-B-multiple prefix the bulk copy moves
+    auto rows_of = [&](const TileInfo &ti) {
+      const int r = ti.count - (int)(rank * 128);
+      return (uint32_t)(r < 0 ? 0 : (r > 128 ? 128 : r));
+    };
+    auto issue = [&](int64_t t, uint32_t buf) {  // one thread
+      const TileInfo ti = tile_info<PREC>(ts, t);
+      const uint32_t bulk = (rows_of(ti) * row_bytes) & ~15u;
+      if (bulk) {
+        ptx::mbar_arrive_expect_tx(bar(B_SFULL + buf), bulk);
+        ptx::bulk_g2s(sbase + L.stage + buf * kStageBytes(PREC),
+                      stage_src + (size_t)(ti.begin + rank * 128) * row_bytes, bulk,
+                      bar(B_SFULL + buf));
+      } else {
+        ptx::mbar_arrive(bar(B_SFULL + buf));
+      }
+    };
+    if (staged && d == 0) {
+      if (t_begin < t_end) issue(t_begin, 0);
+      if (t_begin + 1 < t_end) issue(t_begin + 1, 1);
+    }
     int64_t it = 0;
     for (int64_t t = t_begin; t < t_end; ++t, ++it) {
       const TileInfo ti = tile_info<PREC>(ts, t);
       const uint32_t xb = (uint32_t)(it & 1);
-      uint32_t rec[2][9];
-      bool valid[2];
-      // NN tiles (one tensor-core layer) are digitiser-bound: gather first, then wait.
-      // Deeper nets keep the X-empty wait first (measured 1.7% faster for NN+2: the gather
-      // then lands while the epilogues are busy rather than while the MMA waits on X).
-      const bool early = ti.nh == 1;
-      if (!early) {
-        ptx::mbar_wait(bar(B_XEMPTY + xb), (uint32_t)(((it >> 1) & 1) ^ 1));
-        LAKE_TEV(T_XEMPTY, it, 0, 0);
-      }
+      const uint32_t rows = rows_of(ti);
+      // the row's 32 K values (31 digits + the zero pad), per half (rows d and d + 64)
+      uint32_t dg[2][32];
+      if (staged) {
+        const uint32_t sb = (uint32_t)(it & 1);
+#ifdef LAKE_DIG_SLEEP
+        ptx::mbar_wait_sleep(bar(B_SFULL + sb), (uint32_t)((it >> 1) & 1));
+#else
+        ptx::mbar_wait(bar(B_SFULL + sb), (uint32_t)((it >> 1) & 1));
+#endif
+        LAKE_TEV(T_XEMPTY, it, 1, 0);
+        const uint32_t bulk = (rows * row_bytes) & ~15u;
+        const uint8_t *st = smem + L.stage + sb * kStageBytes(PREC);
 #pragma unroll
-      for (int half = 0; half < 2; ++half) {
-        const int pos = (int)(rank * 128 + d + 64 * half);
-        valid[half] = pos < ti.count;
-        const int64_t p = ti.begin + (valid[half] ? pos : 0);
-        const int64_t io = ts.perm ? (int64_t)ts.perm[p] : p;
-        if (IN_KIND == LAKE_IN_RAW) {
-          const uint32_t *src = reinterpret_cast<const uint32_t *>(in) + io * 9;
+        for (int half = 0; half < 2; ++half) {
+          const uint32_t r = d + 64 * half;
 #pragma unroll
-          for (int f = 0; f < 9; ++f) rec[half][f] = valid[half] ? __ldg(src + f) : 0u;
-        } else {
-          const uint4 *src = reinterpret_cast<const uint4 *>(
-              reinterpret_cast<const uint8_t *>(in) + io * 32);
-          uint4 v0 = make_uint4(0, 0, 0, 0), v1 = v0;
-          if (valid[half]) {
-            v0 = __ldg(src);
-            v1 = __ldg(src + 1);
+          for (int i = 0; i < 32; ++i) dg[half][i] = 0;
+          if (r >= rows) continue;
+          if (ts.pdig) {
+            const uint4 v = *reinterpret_cast<const uint4 *>(st + r * 16);
+            const uint32_t x[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+            for (int k = 0; k < 31; ++k) dg[half][k] = (x[k >> 3] >> (4 * (k & 7))) & 0xFu;
+          } else if (IN_KIND == LAKE_IN_RAW) {
+            uint32_t rec[9];
+            if ((r + 1) * 36 <= bulk) {
+              const uint32_t *src = reinterpret_cast<const uint32_t *>(st + r * 36);
+#pragma unroll
+              for (int f = 0; f < 9; ++f) rec[f] = src[f];
+            } else {  // tail rows past the 16-B-multiple prefix: straight from global
+              const uint32_t *src = reinterpret_cast<const uint32_t *>(in) +
+                                    (size_t)(ti.begin + rank * 128 + r) * 9;
+#pragma unroll
+              for (int f = 0; f < 9; ++f) rec[f] = __ldg(src + f);
+            }
+            digitize_record(rec, [&](int k, uint32_t v) { dg[half][k] = v; });
+          } else {
+            const uint4 v0 = *reinterpret_cast<const uint4 *>(st + r * 32);
+            const uint4 v1 = *reinterpret_cast<const uint4 *>(st + r * 32 + 16);
+            const uint32_t x[8] = {v0.x, v0.y, v0.z, v0.w, v1.x, v1.y, v1.z, v1.w};
+#pragma unroll
+            for (int k = 0; k < 31; ++k) dg[half][k] = (x[k >> 2] >> ((k & 3) * 8)) & 0xFFu;
           }
-          rec[half][0] = v0.x; rec[half][1] = v0.y; rec[half][2] = v0.z; rec[half][3] = v0.w;
-          rec[half][4] = v1.x; rec[half][5] = v1.y; rec[half][6] = v1.z; rec[half][7] = v1.w;
         }
-      }
-      if (early) {
+#ifdef LAKE_DIG_SLEEP
+        ptx::mbar_wait_sleep(bar(B_XEMPTY + xb), (uint32_t)(((it >> 1) & 1) ^ 1));
+#else
         ptx::mbar_wait(bar(B_XEMPTY + xb), (uint32_t)(((it >> 1) & 1) ^ 1));
+#endif
         LAKE_TEV(T_XEMPTY, it, 0, 0);
+      } else {
+        // gather fallback: both rows' loads are issued before any shared store (the
+        // st.shared asm carries a memory clobber, so later loads could not be hoisted)
+        uint32_t rec[2][9];
+        // NN tiles (one tensor-core layer) are digitiser-bound: gather first, then wait.
+        const bool early = ti.nh == 1;
+        if (!early) ptx::mbar_wait(bar(B_XEMPTY + xb), (uint32_t)(((it >> 1) & 1) ^ 1));
+#pragma unroll
+        for (int half = 0; half < 2; ++half) {
+          const uint32_t r = d + 64 * half;
+          const bool valid = r < rows;
+          const int64_t p = ti.begin + rank * 128 + (valid ? r : 0);
+          const int64_t io = ts.perm ? (int64_t)ts.perm[p] : p;
+          if (IN_KIND == LAKE_IN_RAW) {
+            const uint32_t *src = reinterpret_cast<const uint32_t *>(in) + io * 9;
+#pragma unroll
+            for (int f = 0; f < 9; ++f) rec[half][f] = valid ? __ldg(src + f) : 0u;
+          } else {
+            const uint4 *src = reinterpret_cast<const uint4 *>(
+                reinterpret_cast<const uint8_t *>(in) + io * 32);
+            uint4 v0 = make_uint4(0, 0, 0, 0), v1 = v0;
+            if (valid) {
+              v0 = __ldg(src);
+              v1 = __ldg(src + 1);
+            }
+            rec[half][0] = v0.x; rec[half][1] = v0.y; rec[half][2] = v0.z; rec[half][3] = v0.w;
+            rec[half][4] = v1.x; rec[half][5] = v1.y; rec[half][6] = v1.z; rec[half][7] = v1.w;
+            rec[half][8] = 0;
+          }
+        }
+        if (early) ptx::mbar_wait(bar(B_XEMPTY + xb), (uint32_t)(((it >> 1) & 1) ^ 1));
+        LAKE_TEV(T_XEMPTY, it, 0, 0);
+#pragma unroll
+        for (int half = 0; half < 2; ++half) {
+#pragma unroll
+          for (int i = 0; i < 32; ++i) dg[half][i] = 0;
+          if (d + 64 * half >= rows) continue;
+          if (IN_KIND == LAKE_IN_RAW) {
+            digitize_record(rec[half], [&](int k, uint32_t v) { dg[half][k] = v; });
+          } else {
+#pragma unroll
+            for (int k = 0; k < 31; ++k) dg[half][k] = (rec[half][k >> 2] >> ((k & 3) * 8)) & 0xFFu;
+          }
+        }
       }
       const uint32_t xs = sbase + L.x + xb * kXB;
 #pragma unroll
       for (int half = 0; half < 2; ++half) {
         const uint32_t r = d + 64 * half;
-        // the row's 32 K values (31 digits + the zero pad) in the operand type
-        uint32_t dg[32];
-#pragma unroll
-        for (int i = 0; i < 32; ++i) dg[i] = 0;
-        if (valid[half]) {
-          if (IN_KIND == LAKE_IN_RAW) {
-            digitize_record(rec[half], [&](int k, uint32_t v) { dg[k] = v; });
-          } else {
-#pragma unroll
-            for (int k = 0; k < 31; ++k) dg[k] = (rec[half][k >> 2] >> ((k & 3) * 8)) & 0xFFu;
-          }
-        }
         if constexpr (PREC == 2) {
           // tf32 = fp32 bits: 0x4B000000 | v is the float 2^23 + v, exact for v < 2^23, so
           // one subtract of 2^23 gives v exactly (digits 0..9, digit bytes 0..255)
           uint32_t w[32];
 #pragma unroll
           for (int k = 0; k < 32; ++k)
-            w[k] = __float_as_uint(__uint_as_float(0x4B000000u | dg[k]) - 8388608.0f);
+            w[k] = __float_as_uint(__uint_as_float(0x4B000000u | dg[half][k]) - 8388608.0f);
 #pragma unroll
           for (int kg = 0; kg < 8; ++kg)
             ptx::st_shared_v4(xs + kg * kLboR128 + r * 16, w[kg * 4 + 0], w[kg * 4 + 1],
@@ -684,11 +775,11 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
 #pragma unroll
           for (int pp = 0; pp < 16; ++pp) {
             if (IN_KIND == LAKE_IN_RAW || PREC == 0) {
-              const uint32_t u = dg[2 * pp] | (dg[2 * pp + 1] << 16) | kMagic2;
+              const uint32_t u = dg[half][2 * pp] | (dg[half][2 * pp + 1] << 16) | kMagic2;
               w[pp] = PREC == 0 ? ptx::sub_f16x2(u, kMagic2) : ptx::sub_bf16x2(u, kMagic2);
             } else {
-              w[pp] = (uint32_t)__bfloat16_as_ushort(__uint2bfloat16_rn(dg[2 * pp])) |
-                      ((uint32_t)__bfloat16_as_ushort(__uint2bfloat16_rn(dg[2 * pp + 1])) << 16);
+              w[pp] = (uint32_t)__bfloat16_as_ushort(__uint2bfloat16_rn(dg[half][2 * pp])) |
+                      ((uint32_t)__bfloat16_as_ushort(__uint2bfloat16_rn(dg[half][2 * pp + 1])) << 16);
             }
           }
 #pragma unroll
@@ -698,8 +789,11 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         }
       }
       ptx::fence_proxy_async_smem();
-      ptx::named_bar_sync(1, 64);
-      if (d == 0) ptx::mbar_arrive_cluster(xfull_leader0 + xb * 8);
+      ptx::named_bar_sync(1, 64);  // X written; staging buffer it&1 fully read
+      if (d == 0) {
+        ptx::mbar_arrive_cluster(xfull_leader0 + xb * 8);
+        if (staged && t + 2 < t_end) issue(t + 2, (uint32_t)(it & 1));
+      }
       LAKE_TEV(T_XARRIVE, it, 0, 0);
     }
   } else if (warp >= kWarpEpi && warp < kWarpEpi + kEpiWarps) {
@@ -810,7 +904,13 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
             LAKE_TEV(T_LDWAIT, it, l, kc);
           }
         } else {
-          // last hidden layer: fold the 2-neuron output layer (fp32, CUDA cores)
+          // last hidden layer: fold the 2-neuron output layer (fp32, CUDA cores). The row's
+          // output index is loaded first: with model-grouped staged inputs nothing else has
+          // touched perm, so its (DRAM) latency would otherwise sit between the last TMEM
+          // read and the accumulator release.
+          const int pos = (int)(rank * 128 + row);
+          const int64_t pp = ti.begin + pos;
+          const int64_t io = (ts.perm && pos < ti.count) ? (int64_t)__ldg(ts.perm + pp) : pp;
           float p[4] = {0.0f, 0.0f, 0.0f, 0.0f};
 #pragma unroll
           for (uint32_t j = 0; j < kWarpChunks; ++j) {
@@ -832,6 +932,10 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
             }
           }
 #undef EPI_H
+          // accumulator b fully read: release it before the reduction and the output stores
+          ptx::tc_fence_before();
+          __syncwarp();
+          if (lane == 0) ptx::mbar_arrive_cluster(tempty_leader0 + b * 8);
           float p0 = p[0] + p[2], p1 = p[1] + p[3];
           // combine the kEpiPerQ warps of this quadrant (slices hh = 1.. write partials)
           if (hh > 0) {
@@ -853,10 +957,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           if (hh == 0) {
             const float l0 = p0 + wo[2 * kHidden + 0];
             const float l1 = p1 + wo[2 * kHidden + 1];
-            const int pos = (int)(rank * 128 + row);
             if (pos < ti.count) {
-              const int64_t pp = ti.begin + pos;
-              const int64_t io = ts.perm ? (int64_t)ts.perm[pp] : pp;
               if (logits) {
                 logits[io * 2 + 0] = l0;
                 logits[io * 2 + 1] = l1;
@@ -865,10 +966,11 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
             }
           }
         }
-        // accumulator b fully read by this warp
-        ptx::tc_fence_before();
-        __syncwarp();
-        if (lane == 0) ptx::mbar_arrive_cluster(tempty_leader0 + b * 8);
+        if (!last) {  // accumulator b fully read by this warp (the last layer released it above)
+          ptx::tc_fence_before();
+          __syncwarp();
+          if (lane == 0) ptx::mbar_arrive_cluster(tempty_leader0 + b * 8);
+        }
         LAKE_TEV(T_LAYER_END, it, l, warp);
       }
     }
