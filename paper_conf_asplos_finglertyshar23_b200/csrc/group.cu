@@ -28,7 +28,7 @@ constexpr int kBins = LAKE_MAX_MODELS + 1;  // model slots + "unknown"
 
 struct WsHeader {
   int32_t counts[LAKE_MAX_MODELS];
-  int32_t cursor[LAKE_MAX_MODELS];
+  int32_t cursor_unused[LAKE_MAX_MODELS];  // (cursors live in WsLayout::cursor, padded)
   int32_t offsets[LAKE_MAX_MODELS];
   int32_t tile_off64[LAKE_MAX_MODELS + 1];
   int32_t tile_off256[LAKE_MAX_MODELS + 1];
@@ -48,8 +48,10 @@ struct WsHeader {
 
 __host__ __device__ inline size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
 
+constexpr int kCursorStride = 32;  // int32 per cursor (128 B)
+
 struct WsLayout {
-  size_t header, perm, t64_model, t64_begin, t64_count, t256_model, t256_begin, t256_count,
+  size_t cursor, header, perm, t64_model, t64_begin, t64_count, t256_model, t256_begin, t256_count,
       chunk_counts, pdig, total;
   int64_t max64, max256;
 };
@@ -69,6 +71,10 @@ WsLayout ws_layout(int64_t n) {
   L.t256_count = off; off = align256(off + (size_t)L.max256 * 4);
   // per-chunk histograms written by group_hist, read back by group_scatter (no recount)
   L.chunk_counts = off; off = align256(off + (size_t)((n + kChunk - 1) / kChunk) * kBins * 4);
+  // per-model scatter cursors, one 128-B line each: every chunk reserves its range of each
+  // model with a global atomic, and 64 models' cursors packed into 2 lines serialised ~130K
+  // atomics on those lines (the scatter ran at half of HBM bandwidth)
+  L.cursor = off; off = align256(off + (size_t)kBins * kCursorStride * 4);
   // packed digit rows (16 B per I/O) in model-grouped order, for the tensor-core kernel's
   // contiguous bulk-copy staging
   L.pdig = off; off = align256(off + (size_t)n * 16);
@@ -123,8 +129,17 @@ group_hist(const IdT *__restrict__ ids, int64_t n, WsHeader *h,
     for (int i = threadIdx.x; i <= LAKE_MAX_MODELS; i += kGBlock) cnt[i] = 0;
     __syncthreads();
     const int64_t end = (base + kChunk) < n ? base + kChunk : n;
-    for (int64_t i = base + threadIdx.x; i < end; i += kGBlock)
-      atomicAdd(&cnt[bin_of(known_s, (int32_t)__ldg(ids + i))], 1);
+    for (int64_t i0 = base + threadIdx.x; i0 < end; i0 += 4 * kGBlock) {
+      int32_t idv[4];  // four loads in flight per thread
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int64_t i = i0 + (int64_t)u * kGBlock;
+        idv[u] = i < end ? (int32_t)__ldg(ids + i) : 0;
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+        if (i0 + (int64_t)u * kGBlock < end) atomicAdd(&cnt[bin_of(known_s, idv[u])], 1);
+    }
     __syncthreads();
     int32_t *cc = chunk_counts + (base / kChunk) * kBins;
     for (int m = threadIdx.x; m < kBins; m += kGBlock) cc[m] = cnt[m];
@@ -164,14 +179,14 @@ __device__ int32_t block_excl_scan(int32_t v, int32_t *warp_tot, int32_t *total)
 }
 
 __global__ void __launch_bounds__(LAKE_MAX_MODELS)
-group_scan(WsHeader *h) {
+group_scan(WsHeader *h, int32_t *cursor) {
   __shared__ int32_t warp_tot[32];
   __shared__ int32_t total;
   const int m = threadIdx.x;
   const int32_t c = h->counts[m];
   const int32_t off = block_excl_scan(c, warp_tot, &total);
   h->offsets[m] = off;
-  h->cursor[m] = off;
+  cursor[m * kCursorStride] = off;
   const int32_t n_known = total;
   const int32_t t64 = block_excl_scan((c + kF32TileM - 1) / kF32TileM, warp_tot, &total);
   h->tile_off64[m] = t64;
@@ -180,7 +195,7 @@ group_scan(WsHeader *h) {
   h->tile_off256[m] = t256;
   if (m == 0) {
     h->n_known = n_known;
-    h->unk_cursor = n_known;
+    cursor[LAKE_MAX_MODELS * kCursorStride] = n_known;
     h->n_tiles64 = tot64;
     h->n_tiles256 = total;
     h->tile_off64[LAKE_MAX_MODELS] = tot64;
@@ -194,7 +209,7 @@ template <typename IdT, int IN_KIND>
 __global__ void __launch_bounds__(kGBlock)
 group_scatter(const IdT *__restrict__ ids, int64_t n, WsHeader *h, int32_t *__restrict__ perm,
               const int32_t *__restrict__ chunk_counts, const void *__restrict__ in,
-              uint4 *__restrict__ pdig) {
+              uint4 *__restrict__ pdig, int32_t *__restrict__ cursor) {
   __shared__ int32_t cnt[LAKE_MAX_MODELS + 1];
   __shared__ int32_t basep[LAKE_MAX_MODELS + 1];
   __shared__ uint8_t known_s[LAKE_MAX_MODELS];
@@ -206,7 +221,7 @@ group_scatter(const IdT *__restrict__ ids, int64_t n, WsHeader *h, int32_t *__re
     const int64_t end = (base + kChunk) < n ? base + kChunk : n;
     for (int m = threadIdx.x; m <= LAKE_MAX_MODELS; m += kGBlock) {
       const int32_t c = cnt[m];
-      if (c) basep[m] = atomicAdd(m < LAKE_MAX_MODELS ? &h->cursor[m] : &h->unk_cursor, c);
+      if (c) basep[m] = atomicAdd(&cursor[m * kCursorStride], c);
       cnt[m] = 0;
     }
     __syncthreads();
@@ -308,6 +323,7 @@ struct GroupPtrs {
   int64_t max[2];
   int32_t *cc;  // per-chunk histograms
   uint4 *pdig;  // packed digit rows, grouped order
+  int32_t *cursor;  // padded per-model scatter cursors
 };
 
 static GroupPtrs group_ptrs(void *ws, int64_t n) {
@@ -324,6 +340,7 @@ static GroupPtrs group_ptrs(void *ws, int64_t n) {
   p.tc[1] = reinterpret_cast<int32_t *>(b + L.t256_count);
   p.cc = reinterpret_cast<int32_t *>(b + L.chunk_counts);
   p.pdig = reinterpret_cast<uint4 *>(b + L.pdig);
+  p.cursor = reinterpret_cast<int32_t *>(b + L.cursor);
   p.nt[0] = &p.h->n_tiles64;
   p.nt[1] = &p.h->n_tiles256;
   p.max[0] = L.max64;
@@ -344,7 +361,8 @@ cudaError_t launch_group(int64_t n, const void *model_ids, int id_kind, const De
     sms_cache[dev & 63].store(sms, std::memory_order_relaxed);
   }
   const int64_t chunks = (n + kChunk - 1) / kChunk;
-  const int grid = (int)(chunks < 2 * sms ? chunks : 2 * sms);
+  // 4 blocks of 512 threads per SM: full occupancy (32 registers), enough loads in flight
+  const int grid = (int)(chunks < 4 * sms ? chunks : 4 * sms);
   auto hist = [&](auto *ids) {
     if (grid > 0) group_hist<<<grid, kGBlock, 0, s>>>(ids, n, p.h, p.cc);
   };
@@ -352,17 +370,20 @@ cudaError_t launch_group(int64_t n, const void *model_ids, int id_kind, const De
     using IdT = std::remove_cv_t<std::remove_pointer_t<decltype(ids)>>;
     if (grid <= 0) return;
     if (!in)
-      group_scatter<IdT, -1><<<grid, kGBlock, 0, s>>>(ids, n, p.h, p.perm, p.cc, nullptr, nullptr);
+      group_scatter<IdT, -1><<<grid, kGBlock, 0, s>>>(ids, n, p.h, p.perm, p.cc, nullptr, nullptr,
+                                                      p.cursor);
     else if (in_kind == LAKE_IN_RAW)
-      group_scatter<IdT, LAKE_IN_RAW><<<grid, kGBlock, 0, s>>>(ids, n, p.h, p.perm, p.cc, in, p.pdig);
+      group_scatter<IdT, LAKE_IN_RAW><<<grid, kGBlock, 0, s>>>(ids, n, p.h, p.perm, p.cc, in, p.pdig,
+                                                               p.cursor);
     else
-      group_scatter<IdT, LAKE_IN_DIGITS><<<grid, kGBlock, 0, s>>>(ids, n, p.h, p.perm, p.cc, in, p.pdig);
+      group_scatter<IdT, LAKE_IN_DIGITS><<<grid, kGBlock, 0, s>>>(ids, n, p.h, p.perm, p.cc, in,
+                                                                  p.pdig, p.cursor);
   };
   const int32_t *i32 = static_cast<const int32_t *>(model_ids);
   const uint16_t *u16 = static_cast<const uint16_t *>(model_ids);
   const uint8_t *u8 = static_cast<const uint8_t *>(model_ids);
   if (id_kind == 1) hist(u16); else if (id_kind == 2) hist(u8); else hist(i32);
-  group_scan<<<1, LAKE_MAX_MODELS, 0, s>>>(p.h);
+  group_scan<<<1, LAKE_MAX_MODELS, 0, s>>>(p.h, p.cursor);
   if (id_kind == 1) scatter(u16); else if (id_kind == 2) scatter(u8); else scatter(i32);
   const int64_t mt = p.max[0] > p.max[1] ? p.max[0] : p.max[1];
   group_tiles<<<(unsigned)((mt + 255) / 256), 256, 0, s>>>(p.h, p.max[0], p.max[1], p.tm[0],
