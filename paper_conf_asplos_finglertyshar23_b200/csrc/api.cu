@@ -152,9 +152,15 @@ void build_tc_image(const BlobView &v, int prec, uint8_t *img /* 2 * bytes */, s
       const uint32_t u = to_bits(val, prec);
       std::memcpy(base + off, &u, eb);  // little endian: the low eb bytes
     };
+    // layer 0 in the tensor-core K order: slot k holds digit tc_slot_digit(k) (lake_internal.h);
+    // slot 31 holds b0, multiplied by the constant 1 the digitisers put in X's slot 31, so the
+    // MMA adds layer 0's bias and its epilogue is only ReLU + rounding
     for (int n = 0; n < 128; ++n)
-      for (int k = 0; k < kTcK0; ++k)
-        put(umma_off(n, k, 128, eb), k < 31 ? v.W[0][(size_t)(rank * 128 + n) * 31 + k] : 0.0f);
+      for (int k = 0; k < kTcK0; ++k) {
+        const int dgt = tc_slot_digit(k);
+        const size_t row = (size_t)(rank * 128 + n);
+        put(umma_off(n, k, 128, eb), dgt < 31 ? v.W[0][row * 31 + dgt] : v.b[0][row]);
+      }
     for (int l = 1; l < nh; ++l) {
       const size_t o = tc_w0_half_bytes(prec) + (size_t)(l - 1) * tc_wh_half_bytes(prec);
       for (int n = 0; n < 128; ++n)

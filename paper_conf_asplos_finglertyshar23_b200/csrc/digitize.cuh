@@ -11,6 +11,8 @@
 #pragma once
 #include <cstdint>
 
+#include "lake_internal.h"
+
 namespace lake {
 
 // Emit the w digits of min(v, 10^w-1) MSB-first through f(position, digit).
@@ -49,16 +51,18 @@ __device__ __forceinline__ void digitize_record(const uint32_t (&rec)[9], F &&f)
 
 namespace lake {
 
-// Packed digit row (internal workspace format, 16 B per I/O): digit k (0..30) in the nibble
-// (k & 1) of byte k/2 (low nibble first); nibble 31 is 0. Written by the grouping pass in
-// model-grouped order so the fused tensor-core kernel can bulk-copy contiguous rows.
-__device__ __forceinline__ uint4 pack_digits(const uint32_t (&dg)[32]) {
+// Packed digit row (internal workspace format, 16 B per I/O): the digit of tensor-core slot s
+// (tc_slot_digit, lake_internal.h) in nibble (s & 1) of byte s/2 (low nibble first); slot 31
+// is 1 (the layer-0 bias input: W0's slot-31 column holds b0). Written by the grouping pass in model-grouped order so the fused tensor-core kernel
+// can bulk-copy contiguous rows and turn each byte into one operand pair.
+__device__ __forceinline__ uint4 pack_slots(const uint32_t (&dg)[32] /* canonical order */) {
   uint32_t w[4];
 #pragma unroll
   for (int q = 0; q < 4; ++q) {
     uint32_t v = 0;
 #pragma unroll
-    for (int j = 0; j < 8; ++j) v |= (dg[q * 8 + j] & 0xFu) << (4 * j);
+    for (int j = 0; j < 8; ++j)
+      v |= (q * 8 + j == 31 ? 1u : (dg[tc_slot_digit(q * 8 + j)] & 0xFu)) << (4 * j);
     w[q] = v;
   }
   return make_uint4(w[0], w[1], w[2], w[3]);
@@ -70,7 +74,7 @@ __device__ __forceinline__ uint4 pack_record(const uint32_t (&rec)[9]) {
 #pragma unroll
   for (int i = 0; i < 32; ++i) dg[i] = 0;
   digitize_record(rec, [&](int k, uint32_t v) { dg[k] = v; });
-  return pack_digits(dg);
+  return pack_slots(dg);
 }
 
 // Packed row of a LAKE_IN_DIGITS row (bytes 0..30 are digits 0..9).
@@ -79,7 +83,7 @@ __device__ __forceinline__ uint4 pack_digit_bytes(const uint4 lo, const uint4 hi
   uint32_t dg[32];
 #pragma unroll
   for (int k = 0; k < 32; ++k) dg[k] = k < 31 ? (b[k >> 2] >> ((k & 3) * 8)) & 0xFFu : 0u;
-  return pack_digits(dg);
+  return pack_slots(dg);
 }
 
 }  // namespace lake

@@ -55,6 +55,20 @@ __host__ __device__ constexpr uint32_t tc_image_bytes(int nh, int prec = 0) {
 __host__ __device__ constexpr uint32_t tc_resident_bytes(int nh, int prec) {
   return (prec == 2 && nh == 3) ? tc_image_bytes(2, 2) : tc_image_bytes(nh, prec);
 }
+// Layer-0 K order of the tensor-core path (the MMA's reduction order is free, so W0's columns
+// are permuted to match): slot -> canonical digit index. Slots 0-15 are the four
+// 4-digit latency fields, 16-25 the last two digits ("tails") of the five 3-digit queue
+// fields, 26-30 their leading digits ("heads"), 31 the zero pad - so every operand pair of the
+// layer-0 A row is one table lookup (tc digitiser) or one byte of the packed row (nibbles).
+__host__ __device__ constexpr int tc_slot_digit(int s) {
+  return s < 16 ? 3 + s                                   // lat0..lat3: canonical 3..18
+       : s < 26 ? ((s - 16) / 2 == 0 ? 1 : 17 + 3 * ((s - 16) / 2)) + (s & 1)  // tails
+       : s < 31 ? ((s - 26) == 0 ? 0 : 16 + 3 * (s - 26))   // heads: 0, 19, 22, 25, 28
+       : 31;                                                // pad
+}
+static_assert(tc_slot_digit(16) == 1 && tc_slot_digit(17) == 2 && tc_slot_digit(18) == 20 &&
+              tc_slot_digit(25) == 30 && tc_slot_digit(26) == 0 && tc_slot_digit(27) == 19 &&
+              tc_slot_digit(30) == 28 && tc_slot_digit(15) == 18, "tc slot permutation");
 constexpr uint32_t kTcRingSlotBytes = 8192;  // tf32 W2 ring slot: 128 rows x K 16
 constexpr uint32_t kTcRingSlots = 4;
 
@@ -93,9 +107,6 @@ cudaError_t launch_mlp_fp32(const void *in, int in_kind, const TileSched &ts,
                             uint8_t *decisions, float *logits, cudaStream_t s, int device);
 cudaError_t launch_mlp_tc(const void *in, int in_kind, int prec, const TileSched &ts, int nh,
                           uint8_t *decisions, float *logits, cudaStream_t s, int device);
-// two tiles in flight per CTA pair (mlp_tc2.cu): fp16 / bf16 (prec 0 / 1)
-cudaError_t launch_mlp_tc2(const void *in, int in_kind, int prec, const TileSched &ts, int nh,
-                           int grid, uint8_t *decisions, float *logits, cudaStream_t s);
 // Grouping for infer_multi (group.cu).
 size_t group_workspace_bytes(int64_t n);
 int64_t group_max_tiles(int64_t n, int tile_rows);

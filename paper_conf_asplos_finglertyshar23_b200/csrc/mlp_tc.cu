@@ -157,7 +157,7 @@ __host__ __device__ constexpr bool streams_w2(int nh, int prec) {
 __host__ __device__ constexpr uint32_t kStageBytes(int prec) { return prec == 2 ? 2048u : 4608u; }
 
 struct Layout {
-  uint32_t ring, h, x, stage, prm, red, prm0, red0, bar, total;
+  uint32_t ring, h, x, stage, t100, prm, red, prm0, red0, bar, total;
 };
 __host__ __device__ constexpr Layout tc_layout(int nh_layout, int prec) {
   Layout L{};
@@ -165,7 +165,8 @@ __host__ __device__ constexpr Layout tc_layout(int nh_layout, int prec) {
   L.h = L.ring + (streams_w2(nh_layout, prec) ? kTcRingSlots * kTcRingSlotBytes : 0u);
   L.x = L.h + kHBytes;
   L.stage = L.x + 2 * x_bytes(prec);
-  L.prm = L.stage + 2 * kStageBytes(prec);
+  L.t100 = L.stage + 2 * kStageBytes(prec);  // 100 digit pairs (x/10, x%10), operand type
+  L.prm = L.t100 + 100 * (prec == 2 ? 8u : 4u);
   L.red = L.prm + kPrmFloats * 4 + kPrm2Words * 4;
   // group 0's own copy of the output-layer parameters and partial sums: with two epilogue
   // groups, NN tiles (a single layer) are drained by the group of their accumulator buffer
@@ -251,6 +252,9 @@ __host__ __device__ constexpr uint32_t tmem_a_col(uint32_t s) {
 // -> + bias (fp32, one rounding) -> ReLU + one rounding to the operand type -> written back
 // in place into the accumulator it came from (see tmem_a_col), where the next layer's MMA
 // reads it as its A operand (no SMEM H tile, no proxy fence).
+// Layer 0's staged bias is zero: the MMA already added b0 (slot 31 of X is 1, W0's slot-31
+// column is b0: DESIGN.md §2). One code path for every layer keeps the kernel's I-cache
+// footprint down (a second, bias-free variant of the unrolled loops cost 10% at C5).
 template <int PREC, int W>
 __device__ __forceinline__ void epi_to_h_tmem(const uint32_t (&r)[W], const float *bias,
                                               uint32_t col0, uint32_t tlane_base) {
@@ -289,6 +293,101 @@ __device__ __forceinline__ void epi_to_h_tmem(const uint32_t (&r)[W], const floa
   }
 }
 
+// ---- layer-0 A rows in the tensor-core slot order (tc_slot_digit, lake_internal.h) ----------
+// Operand pair (a, b), small integers: the 16-bit pattern M | v is the value M' + v (fp16:
+// 0x6400 = 1024, ulp 1 on [1024, 2048); bf16: 0x4300 = 128, ulp 1 on [128, 256)), so one
+// packed subtract of (M', M') gives (a, b) exactly for a, b < 128.
+template <int PREC>
+__device__ __forceinline__ uint32_t pair_of(uint32_t a, uint32_t b) {
+  constexpr uint32_t kMagic2 = PREC == 0 ? 0x64006400u : 0x43004300u;
+  const uint32_t u = a | (b << 16) | kMagic2;
+  return PREC == 0 ? ptx::sub_f16x2(u, kMagic2) : ptx::sub_bf16x2(u, kMagic2);
+}
+// tf32 (fp32 bits): 0x4B000000 | v is 2^23 + v exactly (v < 2^23), minus 2^23 gives v.
+__device__ __forceinline__ uint32_t tf32_of(uint32_t v) {
+  return __float_as_uint(__uint_as_float(0x4B000000u | v) - 8388608.0f);
+}
+template <int PREC>
+struct XRow {
+  uint32_t w[PREC == 2 ? 32 : 16];  // the row's 32 slots: pairs (fp16/bf16) or values (tf32)
+};
+
+// Raw record -> slot row by table lookups: each 4-digit field is hi = v / 100, lo = v % 100
+// and two entries of the 100-pair table; each 3-digit field contributes its tail pair (lo)
+// and its head digit (hi), heads paired at slots 26-30. D_w(v) = digits of min(v, 10^w - 1).
+template <int PREC>
+__device__ __forceinline__ void row_from_raw(const uint32_t (&rec)[9], const uint32_t *t100,
+                                             XRow<PREC> &x) {
+  uint32_t head[5];
+#pragma unroll
+  for (int f = 0; f < 4; ++f) {  // lat_us[f] -> slots 4f..4f+3
+    const uint32_t v = rec[1 + f] < 9999u ? rec[1 + f] : 9999u;
+    const uint32_t hi = v / 100u, lo = v - 100u * hi;
+    if constexpr (PREC == 2) {
+      x.w[4 * f + 0] = t100[2 * hi]; x.w[4 * f + 1] = t100[2 * hi + 1];
+      x.w[4 * f + 2] = t100[2 * lo]; x.w[4 * f + 3] = t100[2 * lo + 1];
+    } else {
+      x.w[2 * f] = t100[hi];
+      x.w[2 * f + 1] = t100[lo];
+    }
+  }
+#pragma unroll
+  for (int g = 0; g < 5; ++g) {  // q_now, q_hist[0..3] -> tail slots 16+2g, 17+2g; head 26+g
+    const uint32_t r = g == 0 ? rec[0] : rec[4 + g];
+    const uint32_t v = r < 999u ? r : 999u;
+    const uint32_t hi = v / 100u, lo = v - 100u * hi;
+    if constexpr (PREC == 2) {
+      x.w[16 + 2 * g] = t100[2 * lo];
+      x.w[17 + 2 * g] = t100[2 * lo + 1];
+      x.w[26 + g] = tf32_of(hi);
+    } else {
+      x.w[8 + g] = t100[lo];
+    }
+    head[g] = hi;
+  }
+  if constexpr (PREC == 2) {
+    x.w[31] = tf32_of(1);  // slot 31: the constant 1 that multiplies b0
+  } else {
+    x.w[13] = pair_of<PREC>(head[0], head[1]);
+    x.w[14] = pair_of<PREC>(head[2], head[3]);
+    x.w[15] = pair_of<PREC>(head[4], 1);  // slot 31: the constant 1 that multiplies b0
+  }
+}
+// Packed row (slot-order nibbles, digitize.cuh) -> slot row: byte p is the pair of slots 2p,
+// 2p+1.
+template <int PREC>
+__device__ __forceinline__ void row_from_packed(const uint4 v, XRow<PREC> &x) {
+  const uint32_t q[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+  for (int p = 0; p < 16; ++p) {
+    const uint32_t b = (q[p >> 2] >> (8 * (p & 3))) & 0xFFu;
+    if constexpr (PREC == 2) {
+      x.w[2 * p] = tf32_of(b & 0xFu);
+      x.w[2 * p + 1] = tf32_of(b >> 4);
+    } else {
+      x.w[p] = pair_of<PREC>(b & 0xFu, b >> 4);
+    }
+  }
+}
+// Canonical-order values (LAKE_IN_DIGITS bytes; dg[31] = 1, the bias input) -> slot row. Digit bytes can be
+// up to 255: exact in fp16 (< 1024) and tf32; bf16 pairs by conversion instead of the trick.
+template <int PREC>
+__device__ __forceinline__ void row_from_canonical(const uint32_t (&dg)[32], XRow<PREC> &x) {
+#pragma unroll
+  for (int s = 0; s < 32; s += 2) {
+    const uint32_t a = dg[tc_slot_digit(s)], b = dg[tc_slot_digit(s + 1)];
+    if constexpr (PREC == 2) {
+      x.w[s] = tf32_of(a);
+      x.w[s + 1] = tf32_of(b);
+    } else if constexpr (PREC == 0) {
+      x.w[s / 2] = pair_of<0>(a, b);
+    } else {
+      x.w[s / 2] = (uint32_t)__bfloat16_as_ushort(__uint2bfloat16_rn(a)) |
+                   ((uint32_t)__bfloat16_as_ushort(__uint2bfloat16_rn(b)) << 16);
+    }
+  }
+}
+
 // Last hidden layer: ReLU(acc + b) in fp32, accumulated straight into the two logits
 // (two partial sums per logit to halve the dependent-FMA chain).
 template <int W>
@@ -297,9 +396,9 @@ __device__ __forceinline__ void epi_to_logits(const uint32_t (&r)[W], const floa
 #pragma unroll
   for (int c4 = 0; c4 < W / 4; ++c4) {
     const float4 b4 = *reinterpret_cast<const float4 *>(bl + col0 + c4 * 4);
+    const float bb[4] = {b4.x, b4.y, b4.z, b4.w};
     const float4 w0 = *reinterpret_cast<const float4 *>(wo + col0 + c4 * 4);
     const float4 w1 = *reinterpret_cast<const float4 *>(wo + kHidden + col0 + c4 * 4);
-    const float bb[4] = {b4.x, b4.y, b4.z, b4.w};
     const float ww0[4] = {w0.x, w0.y, w0.z, w0.w};
     const float ww1[4] = {w1.x, w1.y, w1.z, w1.w};
 #pragma unroll
@@ -343,6 +442,12 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
                       : (warp == kWarpEpi && rank == 0) ? 1
                       : (warp == kWarpEpi && rank == 1) ? 2
                       : (warp == kWarpEpi + 4 && rank == 0) ? 3 : -1;
+#elif defined(LAKE_TRACE_DIG)  // streams: MMA, digitiser thread 0 of rank 0 / rank 1, epi warp 3
+  int tr_stream = !(tr_buf && cid == 0) ? -1
+                      : (warp == kWarpMma && lane == 0 && rank == 0) ? 0
+                      : (threadIdx.x == 0 && rank == 0) ? 1
+                      : (threadIdx.x == 0 && rank == 1) ? 2
+                      : (warp == kWarpEpi && lane == 0 && rank == 0) ? 3 : -1;
 #else
   int tr_stream = !(tr_buf && cid == 0 && rank == 0) ? -1
                       : (warp == kWarpMma && lane == 0) ? 0 : (warp == kWarpEpi && lane == 0) ? 1
@@ -351,7 +456,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
   uint32_t tr_i = 0;
 #ifdef LAKE_TRACE_SMEM
   const uint32_t tr_smem = sbase + L.total;
-  if (tr_buf && cid == 0 && rank == 0)  // clear the log (keys 0 = unused)
+  if (tr_buf && cid == 0)  // clear the log (keys 0 = unused)
     for (uint32_t i = threadIdx.x; i < 4 * LAKE_TRACE_CAP * 4; i += blockDim.x)
       reinterpret_cast<uint32_t *>(smem + L.total)[i] = 0;
   if (PREC == 2) tr_stream = -1;
@@ -385,6 +490,16 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
   if (warp == kWarpLoad) {
     ptx::tmem_alloc_cg2(sbase + L.bar + kTmemSlot, 512);
     ptx::tmem_relinquish_cg2();
+  }
+  // the digitisers' pair table: entry x = (x / 10, x % 10) in the operand type
+  for (uint32_t x = threadIdx.x; x < 100; x += blockDim.x) {
+    uint32_t *t100 = reinterpret_cast<uint32_t *>(smem + L.t100);
+    if constexpr (PREC == 2) {
+      t100[2 * x] = tf32_of(x / 10);
+      t100[2 * x + 1] = tf32_of(x % 10);
+    } else {
+      t100[x] = pair_of<PREC>(x / 10, x % 10);
+    }
   }
   ptx::tc_fence_before();
   ptx::cluster_sync();
@@ -648,13 +763,13 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       if (t_begin < t_end) issue(t_begin, 0);
       if (t_begin + 1 < t_end) issue(t_begin + 1, 1);
     }
+    const uint32_t *t100 = reinterpret_cast<const uint32_t *>(smem + L.t100);
     int64_t it = 0;
     for (int64_t t = t_begin; t < t_end; ++t, ++it) {
       const TileInfo ti = tile_info<PREC>(ts, t);
       const uint32_t xb = (uint32_t)(it & 1);
       const uint32_t rows = rows_of(ti);
-      // the row's 32 K values (31 digits + the zero pad), per half (rows d and d + 64)
-      uint32_t dg[2][32];
+      XRow<PREC> xr[2];  // rows d and d + 64 in the slot order
       if (staged) {
         const uint32_t sb = (uint32_t)(it & 1);
 #ifdef LAKE_DIG_SLEEP
@@ -668,17 +783,16 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
 #pragma unroll
         for (int half = 0; half < 2; ++half) {
           const uint32_t r = d + 64 * half;
-#pragma unroll
-          for (int i = 0; i < 32; ++i) dg[half][i] = 0;
-          if (r >= rows) continue;
+          const bool valid = r < rows;
           if (ts.pdig) {
-            const uint4 v = *reinterpret_cast<const uint4 *>(st + r * 16);
-            const uint32_t x[4] = {v.x, v.y, v.z, v.w};
-#pragma unroll
-            for (int k = 0; k < 31; ++k) dg[half][k] = (x[k >> 3] >> (4 * (k & 7))) & 0xFu;
+            row_from_packed<PREC>(valid ? *reinterpret_cast<const uint4 *>(st + r * 16)
+                                        : make_uint4(0, 0, 0, 0), xr[half]);
           } else if (IN_KIND == LAKE_IN_RAW) {
             uint32_t rec[9];
-            if ((r + 1) * 36 <= bulk) {
+            if (!valid) {
+#pragma unroll
+              for (int f = 0; f < 9; ++f) rec[f] = 0;
+            } else if ((r + 1) * 36 <= bulk) {
               const uint32_t *src = reinterpret_cast<const uint32_t *>(st + r * 36);
 #pragma unroll
               for (int f = 0; f < 9; ++f) rec[f] = src[f];
@@ -688,13 +802,18 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
 #pragma unroll
               for (int f = 0; f < 9; ++f) rec[f] = __ldg(src + f);
             }
-            digitize_record(rec, [&](int k, uint32_t v) { dg[half][k] = v; });
+            row_from_raw<PREC>(rec, t100, xr[half]);
           } else {
-            const uint4 v0 = *reinterpret_cast<const uint4 *>(st + r * 32);
-            const uint4 v1 = *reinterpret_cast<const uint4 *>(st + r * 32 + 16);
+            uint32_t dg[32];
+            uint4 v0 = make_uint4(0, 0, 0, 0), v1 = v0;
+            if (valid) {
+              v0 = *reinterpret_cast<const uint4 *>(st + r * 32);
+              v1 = *reinterpret_cast<const uint4 *>(st + r * 32 + 16);
+            }
             const uint32_t x[8] = {v0.x, v0.y, v0.z, v0.w, v1.x, v1.y, v1.z, v1.w};
 #pragma unroll
-            for (int k = 0; k < 31; ++k) dg[half][k] = (x[k >> 2] >> ((k & 3) * 8)) & 0xFFu;
+            for (int k = 0; k < 32; ++k) dg[k] = k < 31 ? (x[k >> 2] >> ((k & 3) * 8)) & 0xFFu : 1u;
+            row_from_canonical<PREC>(dg, xr[half]);
           }
         }
 #ifdef LAKE_DIG_SLEEP
@@ -737,56 +856,27 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         LAKE_TEV(T_XEMPTY, it, 0, 0);
 #pragma unroll
         for (int half = 0; half < 2; ++half) {
-#pragma unroll
-          for (int i = 0; i < 32; ++i) dg[half][i] = 0;
-          if (d + 64 * half >= rows) continue;
           if (IN_KIND == LAKE_IN_RAW) {
-            digitize_record(rec[half], [&](int k, uint32_t v) { dg[half][k] = v; });
+            row_from_raw<PREC>(rec[half], t100, xr[half]);
           } else {
+            uint32_t dg[32];
 #pragma unroll
-            for (int k = 0; k < 31; ++k) dg[half][k] = (rec[half][k >> 2] >> ((k & 3) * 8)) & 0xFFu;
+            for (int k = 0; k < 32; ++k) dg[k] = k < 31 ? (rec[half][k >> 2] >> ((k & 3) * 8)) & 0xFFu : 1u;
+            row_from_canonical<PREC>(dg, xr[half]);
           }
         }
       }
+      // an absent row (ragged tile) stores zeros (raw: digits of all-zero fields are zero;
+      // gathered invalid rows read 0s above)
       const uint32_t xs = sbase + L.x + xb * kXB;
 #pragma unroll
       for (int half = 0; half < 2; ++half) {
         const uint32_t r = d + 64 * half;
-        if constexpr (PREC == 2) {
-          // tf32 = fp32 bits: 0x4B000000 | v is the float 2^23 + v, exact for v < 2^23, so
-          // one subtract of 2^23 gives v exactly (digits 0..9, digit bytes 0..255)
-          uint32_t w[32];
+        constexpr int NKG = PREC == 2 ? 8 : 4;  // 16-B core-matrix groups per row
 #pragma unroll
-          for (int k = 0; k < 32; ++k)
-            w[k] = __float_as_uint(__uint_as_float(0x4B000000u | dg[half][k]) - 8388608.0f);
-#pragma unroll
-          for (int kg = 0; kg < 8; ++kg)
-            ptx::st_shared_v4(xs + kg * kLboR128 + r * 16, w[kg * 4 + 0], w[kg * 4 + 1],
-                              w[kg * 4 + 2], w[kg * 4 + 3]);
-        } else {
-          // Value pairs converted with packed arithmetic: the 16-bit pattern M | v is the
-          // value M' + v (fp16: 0x6400 = 1024, ulp 1 on [1024, 2048); bf16: 0x4300 = 128,
-          // ulp 1 on [128, 256)), so one packed subtract of (M', M') yields (v0, v1) exactly
-          // for v < 128 - about half the instructions of per-value I2F + packing. Digit bytes
-          // of LAKE_IN_DIGITS input can reach 255, exact in fp16 (< 1024) but not by the bf16
-          // trick, so that case converts value by value.
-          uint32_t w[16];
-          constexpr uint32_t kMagic2 = PREC == 0 ? 0x64006400u : 0x43004300u;
-#pragma unroll
-          for (int pp = 0; pp < 16; ++pp) {
-            if (IN_KIND == LAKE_IN_RAW || PREC == 0) {
-              const uint32_t u = dg[half][2 * pp] | (dg[half][2 * pp + 1] << 16) | kMagic2;
-              w[pp] = PREC == 0 ? ptx::sub_f16x2(u, kMagic2) : ptx::sub_bf16x2(u, kMagic2);
-            } else {
-              w[pp] = (uint32_t)__bfloat16_as_ushort(__uint2bfloat16_rn(dg[half][2 * pp])) |
-                      ((uint32_t)__bfloat16_as_ushort(__uint2bfloat16_rn(dg[half][2 * pp + 1])) << 16);
-            }
-          }
-#pragma unroll
-          for (int kg = 0; kg < 4; ++kg)
-            ptx::st_shared_v4(xs + kg * kLboR128 + r * 16, w[kg * 4 + 0], w[kg * 4 + 1],
-                              w[kg * 4 + 2], w[kg * 4 + 3]);
-        }
+        for (int kg = 0; kg < NKG; ++kg)
+          ptx::st_shared_v4(xs + kg * kLboR128 + r * 16, xr[half].w[kg * 4 + 0],
+                            xr[half].w[kg * 4 + 1], xr[half].w[kg * 4 + 2], xr[half].w[kg * 4 + 3]);
       }
       ptx::fence_proxy_async_smem();
       ptx::named_bar_sync(1, 64);  // X written; staging buffer it&1 fully read
@@ -831,12 +921,15 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         if (do_h) {
           for (uint32_t i = et; i < (uint32_t)(nh - 1) * kHidden / 4; i += NG)
             reinterpret_cast<float4 *>(hbias)[i] =
-                __ldg(reinterpret_cast<const float4 *>(ti.model->b[0]) + i);
+                i < kHidden / 4 ? make_float4(0.0f, 0.0f, 0.0f, 0.0f)  // b0: added by the MMA
+                                : __ldg(reinterpret_cast<const float4 *>(ti.model->b[0]) + i);
         }
         if (do_last || (kEpiGroups == 2 && nh == 1)) {
           const float4 *src = reinterpret_cast<const float4 *>(ti.model->b[nh - 1]);
-          for (uint32_t i = et; i < kPrmFloats / 4; i += NG)
-            reinterpret_cast<float4 *>(prm)[i] = __ldg(src + i);
+          for (uint32_t i = et; i < kPrmFloats / 4; i += NG)  // NN: b0 is added by the MMA
+            reinterpret_cast<float4 *>(prm)[i] = (nh == 1 && i < kHidden / 4)
+                                                     ? make_float4(0.0f, 0.0f, 0.0f, 0.0f)
+                                                     : __ldg(src + i);
         }
         ptx::named_bar_sync(2 + gy, NG);
         cur = ti.model;
@@ -870,7 +963,11 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         const float *bl = prm;  // last-layer bias
         constexpr bool kPrefetch = W <= 32;  // two W-register buffers
         uint32_t ra[W], rb[W];  // rb unused (eliminated) without prefetch
+// (layer 0's staged biases are zero: the MMA added b0; one code path keeps the unrolled
+// chunk loop small - two variants cost ~40% more instructions and I-cache misses)
 #define EPI_H(R) epi_to_h_tmem<PREC, W>(R, hbias + l * kHidden, col0, tbase)
+// (NN: the staged last-layer bias is b0, zeroed at staging because the MMA added it)
+#define EPI_L(R) epi_to_logits<W>(R, bl, wo, col0, p)
         ptx::tmem_ld_cols<W>(tbase + col_of(0), ra);
         ptx::tmem_ld_wait();
         if (!last) {
@@ -920,18 +1017,19 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
                 if (j & 1) ptx::tmem_ld_cols<W>(tbase + col_of(j + 1), ra);
                 else ptx::tmem_ld_cols<W>(tbase + col_of(j + 1), rb);
               }
-              if (j & 1) epi_to_logits<W>(rb, bl, wo, col0, p);
-              else epi_to_logits<W>(ra, bl, wo, col0, p);
+              if (j & 1) EPI_L(rb);
+              else EPI_L(ra);
               if (j + 1 < kWarpChunks) ptx::tmem_ld_wait();
             } else {
               if (j > 0) {
                 ptx::tmem_ld_cols<W>(tbase + col0, ra);
                 ptx::tmem_ld_wait();
               }
-              epi_to_logits<W>(ra, bl, wo, col0, p);
+              EPI_L(ra);
             }
           }
 #undef EPI_H
+#undef EPI_L
           // accumulator b fully read: release it before the reduction and the output stores
           ptx::tc_fence_before();
           __syncwarp();
@@ -984,9 +1082,21 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
     ptx::tmem_dealloc_cg2(tmem, 512);
   }
 #if defined(LAKE_TRACE) && defined(LAKE_TRACE_SMEM)
-  if (PREC != 2 && tr_buf && cid == 0 && rank == 0)
-    for (uint32_t i = threadIdx.x; i < 4 * LAKE_TRACE_CAP * 2; i += blockDim.x)
-      tr_buf[i] = reinterpret_cast<const unsigned long long *>(smem + L.total)[i];
+  // each CTA of cluster 0 copies the streams it recorded (rank 1 only records in
+  // LAKE_TRACE_DIG / LAKE_TRACE_PAIR builds)
+  if (PREC != 2 && tr_buf && cid == 0)
+    for (uint32_t i = threadIdx.x; i < 4 * LAKE_TRACE_CAP * 2; i += blockDim.x) {
+      const unsigned long long v = reinterpret_cast<const unsigned long long *>(smem + L.total)[i];
+      const uint32_t st = i / (LAKE_TRACE_CAP * 2);
+#if defined(LAKE_TRACE_DIG)
+      const bool mine = rank == 1 ? st == 2 : st != 2;
+#elif defined(LAKE_TRACE_PAIR)
+      const bool mine = rank == 1 ? st == 2 : st != 2;
+#else
+      const bool mine = rank == 0;
+#endif
+      if (mine) tr_buf[i] = v;
+    }
 #endif
 }
 
@@ -1051,16 +1161,8 @@ cudaError_t launch_mlp_tc(const void *in, int in_kind, int prec, const TileSched
   const int64_t clusters = ts.n_tiles < max_clusters ? ts.n_tiles : max_clusters;
   if (clusters <= 0) return cudaSuccess;
   const int grid = (int)(clusters * 2);
-  // Every precision runs this file's kernel. LAKE_TC_TWO_TILE=1 selects the experimental
-  // two-tiles-in-flight kernel (mlp_tc2.cu, fp16/bf16) for A/B measurements: parity-green
-  // but slower so far.
-  static const bool two_tile = [] {
-    const char *e = getenv("LAKE_TC_TWO_TILE");
-    return e && e[0] == '1';
-  }();
   cudaError_t e;
-  if (prec < 2 && two_tile) e = launch_mlp_tc2(in, in_kind, prec, ts, nh, grid, decisions, logits, s);
-  else if (prec == 0) e = launch_p<0>(in, in_kind, ts, nh, decisions, logits, s, grid);
+  if (prec == 0) e = launch_p<0>(in, in_kind, ts, nh, decisions, logits, s, grid);
   else if (prec == 1) e = launch_p<1>(in, in_kind, ts, nh, decisions, logits, s, grid);
   else e = launch_p<2>(in, in_kind, ts, nh, decisions, logits, s, grid);
   count_launch();

@@ -6,3 +6,5 @@ echo "exit $?" >> gpurun_out/t_tc.log
 timeout 120 python bench.py --steps 10 --warmup 3 --no-cpu --no-e2e --no-latency > gpurun_out/bench_f16.json 2> gpurun_out/bench_f16.err
 echo "exit $?" >> gpurun_out/bench_f16.err
 timeout 600 python bench.py --mode report > gpurun_out/report.out 2> gpurun_out/report.err
+python scripts/run_single.py C3 f16 0 20 > gpurun_out/nn_single.txt 2>&1
+python scripts/run_single.py C3 f16 2 20 >> gpurun_out/nn_single.txt 2>&1

@@ -15,7 +15,8 @@ from paper_conf_asplos_finglertyshar23_b200 import inputs, lake  # noqa: E402
 KIND = {1: "XFULL", 2: "TEMPTY", 3: "HREADY", 4: "COMMIT", 5: "DFULL", 6: "CHUNK",
         7: "LAYEREND", 8: "XEMPTY", 9: "XARRIVE", 10: "ISSUED", 11: "LDWAIT", 12: "STS",
         13: "FENCE", 14: "TOP", 15: "SCHED", 16: "WREADY", 17: "MMA0", 18: "CX"}
-STREAM = ({0: "mma", 1: "e3r1", 2: "e3r2", 3: "e7r1"} if os.environ.get("LAKE_TRACE_PAIR") else {0: "q0w4", 1: "q1w5", 2: "q2w6", 3: "q3w3"} if os.environ.get("LAKE_TRACE_QUAD") else {0: "mma", 1: "epi4", 2: "epi11", 3: "dig"})
+STREAM = ({0: "mma", 1: "dig0", 2: "dig1", 3: "epi3"} if os.environ.get("LAKE_TRACE_DIG") else
+          {0: "mma", 1: "e3r1", 2: "e3r2", 3: "e7r1"} if os.environ.get("LAKE_TRACE_PAIR") else {0: "q0w4", 1: "q1w5", 2: "q2w6", 3: "q3w3"} if os.environ.get("LAKE_TRACE_QUAD") else {0: "mma", 1: "epi4", 2: "epi11", 3: "dig"})
 CAP = int(os.environ.get("LAKE_TRACE_CAP", 1 << 16))  # 512 for the SMEM-log build (-DLAKE_TRACE_SMEM)
 
 cfg = sys.argv[1] if len(sys.argv) > 1 else "C5"
@@ -31,12 +32,19 @@ dec = torch.empty(n, dtype=torch.uint8, device="cuda")
 wsb = lake.workspace_bytes(n)
 ws = torch.empty(wsb, dtype=torch.uint8, device="cuda")
 flags = lake.LAKE_IN_RAW | lake.PREC_FLAGS[prec]
-lake.infer_multi(x, flags, n, ids, dec, None, ws, wsb)  # warm
+single = len(w["models"]) == 1  # single-model configs: lake_linnos_infer (staged raw rows)
+mid0 = next(iter(w["models"]))
+def call():
+    if single:
+        lake.infer(x, flags, n, mid0, dec, None)
+    else:
+        lake.infer_multi(x, flags, n, ids, dec, None, ws, wsb)
+call()  # warm
 L = lake.lib()
 buf = torch.zeros(4 * CAP * 2, dtype=torch.int64, device="cuda")
 L.lake_trace_set(ctypes.c_void_p(buf.data_ptr()))
 torch.cuda.synchronize()
-lake.infer_multi(x, flags, n, ids, dec, None, ws, wsb)
+call()
 torch.cuda.synchronize()
 L.lake_trace_set(ctypes.c_void_p(0))
 ev = buf.cpu().numpy().view(np.uint64).reshape(4, CAP, 2)
