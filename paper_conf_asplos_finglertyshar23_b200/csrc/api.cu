@@ -51,6 +51,11 @@ size_t g_prof_used = 0;
 
 int nh_of(int32_t arch) { return arch + 1; }
 
+// single-model FP32 calls with at most this many I/Os take the cluster small-batch kernel
+// (measured device time vs the 16-row tile kernel: NN+1/NN+2 faster up to 64 rows; NN only
+// up to 8 - its single 31-wide layer streams quickly through one CTA anyway)
+inline int64_t fp32_small_max(int32_t arch) { return arch == LAKE_ARCH_NN ? 8 : LAKE_SERVER_MAX_BATCH; }
+
 size_t blob_floats(int32_t arch) {
   switch (arch) {
     case LAKE_ARCH_NN: return 256 * 31 + 256 + 2 * 256 + 2;
@@ -327,7 +332,8 @@ int lake_linnos_load_weights(int32_t model_id, int32_t arch, const float *blob, 
   const int nh = v.nh;
   // FP32 image: permuted W^T per hidden layer, biases, Wout, bout.
   const size_t f_w0 = 32 * 256, f_wh = 256 * 256;
-  const size_t f_total = f_w0 + (nh - 1) * f_wh + nh * 256 + 2 * 256 + 4;
+  const size_t f_main = f_w0 + (nh - 1) * f_wh + nh * 256 + 2 * 256 + 4;
+  const size_t f_total = f_main + (size_t)kServerCtas * kServerRankFloats;  // + cluster image
   std::unique_ptr<float[]> f(new (std::nothrow) float[f_total]());
   if (!f) return LAKE_ERR_NOMEM;
   size_t off_wt[kMaxHiddenLayers], off_b[kMaxHiddenLayers], off_wout, off_bout;
@@ -355,6 +361,27 @@ int lake_linnos_load_weights(int32_t model_id, int32_t arch, const float *blob, 
     off_bout = p;
     f[p] = v.b[nh][0];
     f[p + 1] = v.b[nh][1];
+    // cluster image for server.cu: rank r holds output columns [32r, 32r + 32) of every layer
+    for (int r = 0; r < kServerCtas; ++r) {
+      float *q = &f[f_main + (size_t)r * kServerRankFloats];
+      const int c0 = r * kServerSlice;
+      for (int l = 0; l < nh; ++l)
+        for (int j = 0; j < kServerSlice; ++j) q[l * kServerSlice + j] = v.b[l][c0 + j];
+      q += kMaxHiddenLayers * kServerSlice;
+      std::memcpy(q, v.W[nh], 512 * 4);
+      q += 2 * 256;
+      q[0] = v.b[nh][0];
+      q[1] = v.b[nh][1];
+      q += 4;
+      for (int k = 0; k < 31; ++k)
+        for (int j = 0; j < kServerSlice; ++j) q[k * kServerSlice + j] = v.W[0][(size_t)(c0 + j) * 31 + k];
+      q += kInputs * kServerSlice;
+      for (int l = 1; l < nh; ++l)
+        for (int k = 0; k < 256; ++k)
+          for (int j = 0; j < kServerSlice; ++j)
+            q[(size_t)(l - 1) * 256 * kServerSlice + k * kServerSlice + j] =
+                v.W[l][(size_t)(c0 + j) * 256 + k];
+    }
   }
   // tensor-core images, [prec][rank]: fp16, bf16, tf32
   size_t tc_off[3], tc_total = 0;
@@ -395,6 +422,7 @@ int lake_linnos_load_weights(int32_t model_id, int32_t arch, const float *blob, 
   }
   m.wout = fb + off_wout;
   m.bout = fb + off_bout;
+  m.srv = fb + f_main;  // 16-B aligned: f_main is a multiple of 4 floats
   // publish: device table entry, then host mirror; retire the previous buffers. (No
   // device-wide sync: in-flight work on this model is excluded by the header's contract.)
   if (cudaMemcpy(st->table + model_id, &m, sizeof(m), cudaMemcpyHostToDevice) != cudaSuccess) {
@@ -460,6 +488,13 @@ int lake_linnos_infer(const void *in, uint32_t flags, int64_t n, int32_t model_i
   rc = current_model(model_id, &device, &m, nullptr);
   if (rc != LAKE_OK) return rc;
   if ((flags & LAKE_PREC_MASK) == LAKE_PREC_AUTO) check_flags(flags, n, &in_kind, &prec, m.arch);
+  if (prec < 0 && n <= fp32_small_max(m.arch)) {
+    // small batches: one 8-CTA cluster holds the weights across 8 SMs (server.cu), instead of
+    // one CTA streaming every layer's W^T chunk by chunk (~1 L2 round trip per chunk)
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    ProfScope ps(s);
+    return cuda_status(launch_fp32_small(m, in, in_kind, n, decisions, logits, s));
+  }
   TileSched ts;
   std::memset(&ts, 0, sizeof(ts));
   const int rows = prec < 0 ? kF32TileM : kTcTileRows;

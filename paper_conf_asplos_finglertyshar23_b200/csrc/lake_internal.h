@@ -83,7 +83,22 @@ struct DevModel {
   const float *b[kMaxHiddenLayers];
   const float *wout;                  // [2][256]
   const float *bout;                  // [2]
+  // cluster image (server.cu: persistent server and FP32 small-batch kernel): per cluster
+  // rank r < 8, kServerRankFloats floats: b[3][32] | W_out[2][256] | b_out[4] | W0^T[31][32]
+  // | W_l^T[2][256][32], the rank's 32 output columns of every hidden layer
+  const float *srv;
 };
+constexpr int kServerCtas = 8;
+constexpr int kServerSlice = kHidden / kServerCtas;
+constexpr uint32_t kServerRankFloats = kMaxHiddenLayers * kServerSlice + 2 * kHidden + 4 +
+                                       kInputs * kServerSlice +
+                                       (kMaxHiddenLayers - 1) * kHidden * kServerSlice;
+// bytes of a rank's block a model with nh hidden layers uses (a prefix; multiple of 16)
+__host__ __device__ constexpr uint32_t server_block_bytes(int nh) {
+  return 4u * (kMaxHiddenLayers * kServerSlice + 2 * kHidden + 4 + kInputs * kServerSlice +
+               (nh - 1) * kHidden * kServerSlice);
+}
+static_assert(server_block_bytes(1) % 16 == 0 && kServerRankFloats % 4 == 0, "bulk copy sizes");
 
 // Tile schedule. Single-model calls use tile_model == nullptr (all tiles -> `model`) and
 // implicit contiguous tiles; multi-model calls read a device-built grouping.
@@ -133,6 +148,10 @@ size_t capture_workspace_bytes(int64_t n);
 cudaError_t launch_capture(const int64_t *a, const int64_t *c, const int32_t *dev, int64_t n,
                            uint32_t *raw, void *ws, size_t ws_bytes, cudaStream_t s);
 
+// FP32 small-batch kernel (server.cu): one 8-CTA cluster, weights spread over the cluster,
+// n <= LAKE_SERVER_MAX_BATCH rows of device input; same strict-order arithmetic (bit-exact)
+cudaError_t launch_fp32_small(const DevModel &m, const void *in, int in_kind, int64_t n,
+                              uint8_t *dec, float *logits, cudaStream_t s);
 // persistent doorbell server (server.cu)
 struct Server;
 int server_start(const DevModel &m, int device, Server **out);

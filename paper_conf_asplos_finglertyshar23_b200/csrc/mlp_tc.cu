@@ -114,6 +114,10 @@ constexpr uint32_t kEpiWarps = kEpiGroups * kGroupWarps;
 #ifndef LAKE_CHUNKS
 #define LAKE_CHUNKS 8
 #endif
+#ifndef LAKE_EPI_UNROLL  // unroll factor of the epilogue chunk loops (even: register buffers)
+#define LAKE_EPI_UNROLL 8
+#endif
+constexpr int kEpiUnroll = LAKE_EPI_UNROLL;
 constexpr uint32_t kChunks = LAKE_CHUNKS;          // H column chunks per layer (MMA K-chunks)
 constexpr uint32_t kChunkCols = kHidden / kChunks;
 #ifdef LAKE_EPI_INTERLEAVE
@@ -973,7 +977,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         if (!last) {
           // hidden layer feeding another MMA; with two register buffers the TMEM load of the
           // warp's next chunk is in flight while the current one is converted and stored
-#pragma unroll
+#pragma unroll kEpiUnroll
           for (uint32_t j = 0; j < kWarpChunks; ++j) {
             const uint32_t kc = j, col0 = col_of(j);
             if constexpr (kPrefetch) {
@@ -1009,7 +1013,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           const int64_t pp = ti.begin + pos;
           const int64_t io = (ts.perm && pos < ti.count) ? (int64_t)__ldg(ts.perm + pp) : pp;
           float p[4] = {0.0f, 0.0f, 0.0f, 0.0f};
-#pragma unroll
+#pragma unroll kEpiUnroll
           for (uint32_t j = 0; j < kWarpChunks; ++j) {
             const uint32_t col0 = col_of(j);
             if constexpr (kPrefetch) {

@@ -10,6 +10,7 @@
 // column slice, all-gathering activations through distributed shared memory), CTA 0 writes
 // decisions / logits straight into the mailbox and publishes the sequence number back.
 // Arithmetic is the FP32 path's strict order (reading R15): bit-exact with the oracle.
+#include <atomic>
 #include <cstring>
 #include <new>
 
@@ -36,13 +37,16 @@ struct alignas(128) Mailbox {
   unsigned long long t[8];    // phase timestamps of the last batch (%globaltimer, ns)
 };
 
-struct ServerSmem {
-  float w0[kInputs][kSlice];                 // W0^T slice
-  float wh[kMaxHiddenLayers - 1][kHidden][kSlice];  // W_l^T slices, l = 1..nh-1
+// The first five members are, byte for byte, one rank's block of the model's cluster image
+// (api.cu, DevModel::srv): one bulk copy of its used prefix loads a CTA's weights.
+struct alignas(16) ServerSmem {
   float b[kMaxHiddenLayers][kSlice];
   float wout[2][kHidden];
   float bout[4];
-  float act[2][LAKE_SERVER_MAX_BATCH][kActStride];  // all-gathered activations
+  float w0[kInputs][kSlice];                 // W0^T slice
+  float wh[kMaxHiddenLayers - 1][kHidden][kSlice];  // W_l^T slices, l = 1..nh-1
+  unsigned long long wbar, wbar_pad;         // weight bulk-copy completion (16 B: act stays 16-B aligned)
+  alignas(16) float act[2][LAKE_SERVER_MAX_BATCH][kActStride];  // all-gathered activations
   uint32_t rawbuf[LAKE_SERVER_MAX_BATCH * 9 + 4];    // CTA 0: the batch's raw records
   uint32_t seq;
   uint32_t n;
@@ -80,79 +84,96 @@ __device__ __forceinline__ uint4 ld_relaxed_sys_v4(const void *p) {
   return v;
 }
 
+// PERSISTENT: the doorbell server (this file's NEXT-2). !PERSISTENT: the same cluster
+// evaluation launched once for one small batch already in device memory (n <= 64 raw records
+// or digit rows), the FP32 path's small-batch kernel: the weights are spread over 8 SMs and
+// fetched by all of them at once instead of streamed through one CTA layer by layer.
+template <bool PERSISTENT, int IN_KIND>
 __global__ void __cluster_dims__(kCtas, 1, 1) __launch_bounds__(kThreadsS, 1)
 server_kernel(const __grid_constant__ DevModel model, Mailbox *mb, const uint32_t *raw,
-              uint8_t *decisions, float *logits) {
+              uint8_t *decisions, float *logits, uint32_t n_batch) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   ServerSmem &sm = *reinterpret_cast<ServerSmem *>(smem_raw);
   const int tid = threadIdx.x;
   const uint32_t rank = ptx::cluster_ctarank();
   const int col0 = rank * kSlice;
   const int nh = model.nh;
-  // ---- resident weights: this CTA's column slice (the FP32 image stores W^T with permuted
-  // columns; position p(j) = (jj/4)*128 + tc*4 + (jj%4), tc = j%32, jj = j/32)
-  auto pcol = [](int j) { return ((j >> 5) >> 2) * 128 + (j & 31) * 4 + ((j >> 5) & 3); };
-  for (int i = tid; i < kInputs * kSlice; i += kThreadsS) {
-    const int k = i / kSlice, jl = i % kSlice;
-    sm.w0[k][jl] = model.wt[0][k * kHidden + pcol(col0 + jl)];
-  }
-  for (int l = 1; l < nh; ++l)
-    for (int i = tid; i < kHidden * kSlice; i += kThreadsS) {
-      const int k = i / kSlice, jl = i % kSlice;
-      sm.wh[l - 1][k][jl] = model.wt[l][k * kHidden + pcol(col0 + jl)];
+  // ---- resident weights: this CTA's block of the cluster image, one bulk copy (TMA)
+  {
+    const uint32_t wbar = ptx::smem_u32(&sm.wbar);
+    const uint32_t bytes = server_block_bytes(nh);
+    if (tid == 0) {
+      ptx::mbar_init(wbar, 1);
+      ptx::fence_mbar_init();
+      ptx::mbar_arrive_expect_tx(wbar, bytes);
+      ptx::bulk_g2s(ptx::smem_u32(&sm.b[0][0]), model.srv + (size_t)rank * kServerRankFloats,
+                    bytes, wbar);
     }
-  for (int i = tid; i < nh * kSlice; i += kThreadsS)
-    sm.b[i / kSlice][i % kSlice] = model.b[i / kSlice][col0 + i % kSlice];
-  for (int i = tid; i < 2 * kHidden; i += kThreadsS) sm.wout[i / kHidden][i % kHidden] = model.wout[i];
-  if (tid < 2) sm.bout[tid] = model.bout[tid];
+    __syncthreads();
+    ptx::mbar_wait(wbar, 0);
+  }
   uint32_t act_remote[kCtas];  // shared::cluster address of act[0][0][0] in every CTA
   for (int c = 0; c < kCtas; ++c) act_remote[c] = ptx::mapa(ptx::smem_u32(&sm.act[0][0][0]), c);
   constexpr uint32_t kActBuf = LAKE_SERVER_MAX_BATCH * kActStride * 4;
   uint32_t last = 0;
   ptx::cluster_sync();
-  if (rank == 0 && tid == 0) {  // weights resident: tell server_start it may return
+  if (PERSISTENT && rank == 0 && tid == 0) {  // weights resident: server_start may return
     __threadfence_system();
     st_release_sys(&mb->seq_out, kReady);
   }
 
   for (;;) {
-    // ---- doorbell: CTA 0 / thread 0 polls; everyone else sleeps in the cluster barrier
-    if (rank == 0 && tid < 32) {
-      if (tid == 0) {
-        uint32_t s;
-        while ((s = ld_acquire_sys(&mb->seq_in)) == last) __nanosleep(64);
-        SRV_T(0);
-        sm.seq = s;
-        sm.n = mb->n;
+    uint32_t seq0 = 0, n = n_batch;
+    if constexpr (PERSISTENT) {
+      // ---- doorbell: CTA 0 / thread 0 polls; everyone else sleeps in the cluster barrier
+      if (rank == 0 && tid < 32) {
+        if (tid == 0) {
+          uint32_t s;
+          while ((s = ld_acquire_sys(&mb->seq_in)) == last) __nanosleep(64);
+          SRV_T(0);
+          sm.seq = s;
+          sm.n = mb->n;
+        }
+        __syncwarp();  // reconverge before the .aligned cluster barrier
       }
-      __syncwarp();  // reconverge before the .aligned cluster barrier
+      ptx::cluster_sync();
+      // every CTA reads seq/n from CTA 0's shared memory
+      {
+        const uint32_t a_seq = ptx::mapa(ptx::smem_u32(&sm.seq), 0);
+        const uint32_t a_n = ptx::mapa(ptx::smem_u32(&sm.n), 0);
+        asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(seq0) : "r"(a_seq) : "memory");
+        asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(n) : "r"(a_n) : "memory");
+      }
+      if (seq0 == kStop) break;
+      last = seq0;
     }
-    ptx::cluster_sync();
-    // every CTA reads seq/n from CTA 0's shared memory
-    uint32_t seq0, n;
-    {
-      const uint32_t a_seq = ptx::mapa(ptx::smem_u32(&sm.seq), 0);
-      const uint32_t a_n = ptx::mapa(ptx::smem_u32(&sm.n), 0);
-      asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(seq0) : "r"(a_seq) : "memory");
-      asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(n) : "r"(a_n) : "memory");
-    }
-    if (seq0 == kStop) break;
-    last = seq0;
     if (n > LAKE_SERVER_MAX_BATCH) n = LAKE_SERVER_MAX_BATCH;
-    // ---- CTA 0 fetches the batch once (16-byte system-scope loads from the mailbox),
-    // digitises it and broadcasts the digit rows into every CTA's act[0]
+    // ---- CTA 0 fetches the batch once (persistent: 16-byte system-scope loads from the
+    // mailbox), digitises it and broadcasts the digit rows into every CTA's act[0]
     if (rank == 0) {
-      const int n16 = ((int)n * 36 + 15) / 16;
-      for (int i = tid; i < n16; i += kThreadsS)
-        reinterpret_cast<uint4 *>(sm.rawbuf)[i] = ld_relaxed_sys_v4(reinterpret_cast<const uint4 *>(raw) + i);
+      if constexpr (PERSISTENT) {  // the mailbox is padded: whole 16-B vectors
+        const int n16 = ((int)n * 36 + 15) / 16;
+        for (int i = tid; i < n16; i += kThreadsS)
+          reinterpret_cast<uint4 *>(sm.rawbuf)[i] =
+              ld_relaxed_sys_v4(reinterpret_cast<const uint4 *>(raw) + i);
+      } else {  // caller's device buffer: exactly its n rows, 4-B loads
+        const int nw = (int)n * (IN_KIND == LAKE_IN_RAW ? 9 : 8);
+        for (int i = tid; i < nw; i += kThreadsS) sm.rawbuf[i] = __ldg(raw + i);
+      }
       __syncthreads();
       if (tid < (int)n) {
-        uint32_t rec[9];
-#pragma unroll
-        for (int f = 0; f < 9; ++f) rec[f] = sm.rawbuf[tid * 9 + f];
         float dg[32];
         dg[31] = 0.0f;
-        digitize_record(rec, [&](int pos, uint32_t d) { dg[pos] = (float)d; });
+        if constexpr (IN_KIND == LAKE_IN_RAW) {
+          uint32_t rec[9];
+#pragma unroll
+          for (int f = 0; f < 9; ++f) rec[f] = sm.rawbuf[tid * 9 + f];
+          digitize_record(rec, [&](int pos, uint32_t d) { dg[pos] = (float)d; });
+        } else {
+#pragma unroll
+          for (int k = 0; k < 31; ++k)
+            dg[k] = (float)((sm.rawbuf[tid * 8 + (k >> 2)] >> ((k & 3) * 8)) & 0xFFu);
+        }
         const uint32_t off = (uint32_t)(tid * kActStride) * 4;
 #pragma unroll
         for (int c = 0; c < kCtas; ++c)
@@ -227,20 +248,48 @@ server_kernel(const __grid_constant__ DevModel model, Mailbox *mb, const uint32_
           if (c == 0) decisions[r] = (other > z) ? 1 : 0;  // logit1 > logit0; ties/NaN -> 0
         }
       }
-      __syncthreads();
-      if (tid == 0) {
-        SRV_T(5);
-        __threadfence_system();
-        SRV_T(6);
-        st_release_sys(&mb->seq_out, seq0);
+      if constexpr (PERSISTENT) {
+        __syncthreads();
+        if (tid == 0) {
+          SRV_T(5);
+          __threadfence_system();
+          SRV_T(6);
+          st_release_sys(&mb->seq_out, seq0);
+        }
+        __syncwarp();
       }
-      __syncwarp();
     }
+    if constexpr (!PERSISTENT) break;
   }
   ptx::cluster_sync();  // no CTA leaves while a peer may still read its shared memory
 }
 
+template <int IN_KIND>
+cudaError_t small_launch(const DevModel &m, const void *in, int64_t n, uint8_t *dec, float *logits,
+                         cudaStream_t st) {
+  static std::atomic<bool> attr_set[64];  // per device; a race repeats the attribute call
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (!attr_set[dev & 63].load(std::memory_order_acquire)) {
+    cudaError_t e = cudaFuncSetAttribute(server_kernel<false, IN_KIND>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)sizeof(ServerSmem));
+    if (e != cudaSuccess) return e;
+    attr_set[dev & 63].store(true, std::memory_order_release);
+  }
+  server_kernel<false, IN_KIND><<<kCtas, kThreadsS, sizeof(ServerSmem), st>>>(
+      m, nullptr, static_cast<const uint32_t *>(in), dec, logits, (uint32_t)n);
+  return cudaGetLastError();
+}
+
 }  // namespace
+
+cudaError_t launch_fp32_small(const DevModel &m, const void *in, int in_kind, int64_t n,
+                              uint8_t *dec, float *logits, cudaStream_t s) {
+  count_launch();
+  return in_kind == LAKE_IN_RAW ? small_launch<LAKE_IN_RAW>(m, in, n, dec, logits, s)
+                                : small_launch<LAKE_IN_DIGITS>(m, in, n, dec, logits, s);
+}
 
 struct Server {
   int device = 0;
@@ -275,8 +324,8 @@ int server_start(const DevModel &m, int device, Server **out) {
   cudaError_t e = cudaHostGetDevicePointer(&d_host, s->host, 0);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&s->stream, cudaStreamNonBlocking);
   if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(server_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)sizeof(ServerSmem));
+    e = cudaFuncSetAttribute(server_kernel<true, LAKE_IN_RAW>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(ServerSmem));
   if (e != cudaSuccess) {
     release_host(s->host);
     delete s;
@@ -284,10 +333,10 @@ int server_start(const DevModel &m, int device, Server **out) {
   }
   uint8_t *d = static_cast<uint8_t *>(d_host);
   servers_started();  // from here on, library frees defer until the last server stops
-  server_kernel<<<kCtas, kThreadsS, sizeof(ServerSmem), s->stream>>>(
+  server_kernel<true, LAKE_IN_RAW><<<kCtas, kThreadsS, sizeof(ServerSmem), s->stream>>>(
       m, reinterpret_cast<Mailbox *>(d), reinterpret_cast<const uint32_t *>(d + sizeof(Mailbox)),
       d + sizeof(Mailbox) + LAKE_SERVER_MAX_BATCH * 36,
-      reinterpret_cast<float *>(d + sizeof(Mailbox) + LAKE_SERVER_MAX_BATCH * 40));
+      reinterpret_cast<float *>(d + sizeof(Mailbox) + LAKE_SERVER_MAX_BATCH * 40), 0);
   count_launch();
   e = cudaGetLastError();
   // wait until the weights are resident (the model may be unloaded right after we return)

@@ -88,6 +88,25 @@ def test_fp32_digits_input_bit_exact(arch):
     assert np.array_equal(lg.view(np.uint32), rlg.view(np.uint32))
 
 
+@pytest.mark.parametrize("arch", ARCHS)
+@pytest.mark.parametrize("n", [1, 7, 64])
+def test_fp32_small_batch_cluster_kernel(arch, n):
+    """n <= 64 single-model FP32 calls run the 8-CTA cluster kernel (server.cu): bit-exact
+    for raw and digit inputs, with and without logits."""
+    raw = _trace(n, seed=200 + n)
+    rlg, rdec = oracle.infer_raw(arch, inputs.weights(arch, 10 + arch), raw, nthreads=0)
+    lg, dec = run_infer(10 + arch, raw, lake.LAKE_IN_RAW | lake.LAKE_PREC_FP32)
+    assert np.array_equal(dec, rdec)
+    assert np.array_equal(lg.view(np.uint32), rlg.view(np.uint32))
+    dig = np.zeros((n, 32), np.uint8)
+    dig[:, :31] = oracle.digitize(raw)
+    lg2, dec2 = run_infer(10 + arch, dig, lake.LAKE_IN_DIGITS | lake.LAKE_PREC_FP32)
+    assert np.array_equal(dec2, rdec)
+    assert np.array_equal(lg2.view(np.uint32), rlg.view(np.uint32))
+    _, dec3 = run_infer(10 + arch, raw, lake.LAKE_IN_RAW | lake.LAKE_PREC_FP32, logits=False)
+    assert np.array_equal(dec3, rdec)
+
+
 def test_fp32_without_logits():
     raw = _trace(500)
     _, dec = run_infer(12, raw, lake.LAKE_IN_RAW, logits=False)
