@@ -167,10 +167,13 @@ void build_tc_image(const BlobView &v, int prec, uint8_t *img /* 2 * bytes */, s
         put(umma_off(n, k, 128, eb), dgt < 31 ? v.W[0][row * 31 + dgt] : v.b[0][row]);
       }
     for (int l = 1; l < nh; ++l) {
-      const size_t o = tc_w0_half_bytes(prec) + (size_t)(l - 1) * tc_wh_half_bytes(prec);
+      const size_t o = tc_wh_off(l, prec);
       for (int n = 0; n < 128; ++n)
         for (int k = 0; k < 256; ++k)
           put(o + umma_off(n, k, 128, eb), v.W[l][(size_t)(rank * 128 + n) * 256 + k]);
+      if (tc_bias_block_bytes(prec))  // bias block: K column 0 = b_l (the rest stays 0)
+        for (int n = 0; n < 128; ++n)
+          put(o + tc_wh_half_bytes(prec) + umma_off(n, 0, 128, eb), v.b[l][rank * 128 + n]);
     }
   }
 }

@@ -43,11 +43,25 @@ __host__ __device__ constexpr uint32_t tc_wh_half_bytes(int prec) {
 }
 constexpr uint32_t kTcW0HalfBytes = tc_w0_half_bytes(0);
 constexpr uint32_t kTcWhHalfBytes = tc_wh_half_bytes(0);
-// Per-rank weight image: W0 half | hidden-layer halves. The biases and the 2-wide output
-// layer stay fp32 (the epilogue stages them from the FP32 image: b[0] .. b[nh-1],
+// fp16/bf16: each hidden layer l >= 1 is followed by a bias block, 128 rows x K 16 in the
+// operand layout with b_l in K column 0 (zeros elsewhere): one extra MMA with a constant
+// "ones" A tile initialises the accumulator with the bias, so no epilogue adds a bias
+// (layer 0's bias rides in W0's K slot 31). tf32 has no SMEM for the blocks (0 bytes).
+__host__ __device__ constexpr uint32_t tc_bias_block_bytes(int prec) {
+  return prec == 2 ? 0u : 128u * 16u * tc_elem_bytes(prec);  // 4 KB
+}
+// stride between hidden layers in the image, and a hidden layer's offset
+__host__ __device__ constexpr uint32_t tc_layer_stride(int prec) {
+  return tc_wh_half_bytes(prec) + tc_bias_block_bytes(prec);
+}
+__host__ __device__ constexpr uint32_t tc_wh_off(int l, int prec) {
+  return tc_w0_half_bytes(prec) + (l - 1) * tc_layer_stride(prec);
+}
+// Per-rank weight image: W0 half | hidden-layer halves (+ bias blocks). The fp32 biases and
+// the 2-wide output layer are staged by the epilogue from the FP32 image (b[0] .. b[nh-1],
 // W_out[2][256], b_out[2] are contiguous there).
 __host__ __device__ constexpr uint32_t tc_image_bytes(int nh, int prec = 0) {
-  return tc_w0_half_bytes(prec) + (nh - 1) * tc_wh_half_bytes(prec);
+  return tc_w0_half_bytes(prec) + (nh - 1) * tc_layer_stride(prec);
 }
 // Bytes of the per-rank image kept resident in SMEM. Everything, except for tf32 NN+2
 // (272 KB per rank > 227 KB): its last hidden layer (W2, 128 KB per rank) is streamed

@@ -161,7 +161,7 @@ __host__ __device__ constexpr bool streams_w2(int nh, int prec) {
 __host__ __device__ constexpr uint32_t kStageBytes(int prec) { return prec == 2 ? 2048u : 4608u; }
 
 struct Layout {
-  uint32_t ring, h, x, stage, t100, prm, red, prm0, red0, bar, total;
+  uint32_t ring, h, x, stage, t100, ones, prm, red, prm0, red0, bar, total;
 };
 __host__ __device__ constexpr Layout tc_layout(int nh_layout, int prec) {
   Layout L{};
@@ -170,7 +170,8 @@ __host__ __device__ constexpr Layout tc_layout(int nh_layout, int prec) {
   L.x = L.h + kHBytes;
   L.stage = L.x + 2 * x_bytes(prec);
   L.t100 = L.stage + 2 * kStageBytes(prec);  // 100 digit pairs (x/10, x%10), operand type
-  L.prm = L.t100 + 100 * (prec == 2 ? 8u : 4u);
+  L.ones = L.t100 + 100 * (prec == 2 ? 8u : 4u);  // "ones" A tile of the bias MMA (fp16/bf16)
+  L.prm = L.ones + tc_bias_block_bytes(prec);
   L.red = L.prm + kPrmFloats * 4 + kPrm2Words * 4;
   // group 0's own copy of the output-layer parameters and partial sums: with two epilogue
   // groups, NN tiles (a single layer) are drained by the group of their accumulator buffer
@@ -238,9 +239,7 @@ constexpr uint32_t kWarpLoad = 3;
 constexpr uint32_t kWarpEpi = 4;
 #endif
 
-__device__ __forceinline__ uint32_t img_wh(int l, int prec) {
-  return tc_w0_half_bytes(prec) + (l - 1) * tc_wh_half_bytes(prec);
-}
+__device__ __forceinline__ uint32_t img_wh(int l, int prec) { return tc_wh_off(l, prec); }
 
 // Column of TMEM (relative to the H buffer) where K-step s of the next layer's A operand
 // sits. fp16/bf16: the warp's kEpiCols fp32 columns [col0, col0 + kEpiCols) are packed in
@@ -259,6 +258,8 @@ __host__ __device__ constexpr uint32_t tmem_a_col(uint32_t s) {
 // Layer 0's staged bias is zero: the MMA already added b0 (slot 31 of X is 1, W0's slot-31
 // column is b0: DESIGN.md §2). One code path for every layer keeps the kernel's I-cache
 // footprint down (a second, bias-free variant of the unrolled loops cost 10% at C5).
+// fp16/bf16: every bias was added by the MMA (layer 0: W0's slot 31; hidden layers: the
+// bias-block MMA), so the epilogue is ReLU + one rounding. tf32 adds the fp32 bias here.
 template <int PREC, int W>
 __device__ __forceinline__ void epi_to_h_tmem(const uint32_t (&r)[W], const float *bias,
                                               uint32_t col0, uint32_t tlane_base) {
@@ -266,8 +267,11 @@ __device__ __forceinline__ void epi_to_h_tmem(const uint32_t (&r)[W], const floa
   uint32_t p[NW];
 #pragma unroll
   for (int c4 = 0; c4 < W / 4; ++c4) {
-    const float4 b4 = *reinterpret_cast<const float4 *>(bias + col0 + c4 * 4);
-    const float bb[4] = {b4.x, b4.y, b4.z, b4.w};
+    float bb[4] = {0.0f, 0.0f, 0.0f, 0.0f};
+    if constexpr (PREC == 2) {
+      const float4 b4 = *reinterpret_cast<const float4 *>(bias + col0 + c4 * 4);
+      bb[0] = b4.x; bb[1] = b4.y; bb[2] = b4.z; bb[3] = b4.w;
+    }
 #pragma unroll
     for (int e = 0; e < 4; e += 2) {
       const int c = c4 * 4 + e;
@@ -275,8 +279,8 @@ __device__ __forceinline__ void epi_to_h_tmem(const uint32_t (&r)[W], const floa
       if constexpr (PREC == 2) { p[c] = r[c]; p[c + 1] = r[c + 1]; }
       else p[c / 2] = r[c] ^ r[c + 1];
 #else
-      const float v0 = __uint_as_float(r[c]) + bb[e];
-      const float v1 = __uint_as_float(r[c + 1]) + bb[e + 1];
+      const float v0 = PREC == 2 ? __uint_as_float(r[c]) + bb[e] : __uint_as_float(r[c]);
+      const float v1 = PREC == 2 ? __uint_as_float(r[c + 1]) + bb[e + 1] : __uint_as_float(r[c + 1]);
       if constexpr (PREC == 2) {
         p[c] = ptx::relu_tf32(v0);
         p[c + 1] = ptx::relu_tf32(v1);
@@ -393,14 +397,18 @@ __device__ __forceinline__ void row_from_canonical(const uint32_t (&dg)[32], XRo
 }
 
 // Last hidden layer: ReLU(acc + b) in fp32, accumulated straight into the two logits
-// (two partial sums per logit to halve the dependent-FMA chain).
-template <int W>
+// (two partial sums per logit to halve the dependent-FMA chain). fp16/bf16: b is already
+// in acc (bias MMA).
+template <int PREC, int W>
 __device__ __forceinline__ void epi_to_logits(const uint32_t (&r)[W], const float *bl,
                                               const float *wo, uint32_t col0, float (&p)[4]) {
 #pragma unroll
   for (int c4 = 0; c4 < W / 4; ++c4) {
-    const float4 b4 = *reinterpret_cast<const float4 *>(bl + col0 + c4 * 4);
-    const float bb[4] = {b4.x, b4.y, b4.z, b4.w};
+    float bb[4] = {0.0f, 0.0f, 0.0f, 0.0f};
+    if constexpr (PREC == 2) {
+      const float4 b4 = *reinterpret_cast<const float4 *>(bl + col0 + c4 * 4);
+      bb[0] = b4.x; bb[1] = b4.y; bb[2] = b4.z; bb[3] = b4.w;
+    }
     const float4 w0 = *reinterpret_cast<const float4 *>(wo + col0 + c4 * 4);
     const float4 w1 = *reinterpret_cast<const float4 *>(wo + kHidden + col0 + c4 * 4);
     const float ww0[4] = {w0.x, w0.y, w0.z, w0.w};
@@ -410,7 +418,7 @@ __device__ __forceinline__ void epi_to_logits(const uint32_t (&r)[W], const floa
 #ifdef LAKE_ABL_NOLOGITS  // timing-only ablation: no output-layer arithmetic
       p[e] += __uint_as_float(r[c4 * 4 + e]) + bb[e] + ww0[e] + ww1[e];
 #else
-      float h = __uint_as_float(r[c4 * 4 + e]) + bb[e];
+      float h = PREC == 2 ? __uint_as_float(r[c4 * 4 + e]) + bb[e] : __uint_as_float(r[c4 * 4 + e]);
       h = h > 0.0f ? h : 0.0f;
       p[(e & 1) * 2 + 0] = fmaf(h, ww0[e], p[(e & 1) * 2 + 0]);
       p[(e & 1) * 2 + 1] = fmaf(h, ww1[e], p[(e & 1) * 2 + 1]);
@@ -494,6 +502,15 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
   if (warp == kWarpLoad) {
     ptx::tmem_alloc_cg2(sbase + L.bar + kTmemSlot, 512);
     ptx::tmem_relinquish_cg2();
+  }
+  // the bias MMA's A operand (fp16/bf16): 128 rows x K 16, K column 0 = 1, zeros elsewhere
+  if constexpr (PREC != 2) {
+    uint32_t *ones = reinterpret_cast<uint32_t *>(smem + L.ones);
+    constexpr uint32_t kOne = PREC == 0 ? 0x3C00u : 0x3F80u;
+    for (uint32_t i = threadIdx.x; i < tc_bias_block_bytes(PREC) / 4; i += blockDim.x)
+      // core layout: element (r, k) at (k/8)*2048 + r*16 + (k%8)*2; k = 0 <=> word r*4
+      ones[i] = (i < 128 * 4 && (i & 3) == 0) ? kOne : 0u;
+    ptx::fence_proxy_async_smem();  // generic-proxy writes read by the tensor core
   }
   // the digitisers' pair table: entry x = (x / 10, x % 10) in the operand type
   for (uint32_t x = threadIdx.x; x < 100; x += blockDim.x) {
@@ -596,6 +613,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       const uint64_t xdesc1 = ptx::umma_desc(sbase + L.x + kXB, kLboR128, 128);
       const uint64_t w0desc = ptx::umma_desc(sbase, kLboR128, 128);
       const uint64_t ringdesc = ptx::umma_desc(sbase + L.ring, kLboR128, 128);
+      const uint64_t onesdesc = ptx::umma_desc(sbase + L.ones, kLboR128, 128);
       uint64_t whdesc[kMaxHiddenLayers];
       for (int l = 1; l < kMaxHiddenLayers; ++l)
         whdesc[l] = ptx::umma_desc(sbase + img_wh(l, PREC), kLboR128, 128);
@@ -674,6 +692,12 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           const uint32_t ha = tm + ((g - 1) & 1) * 256;
           const bool from_ring = stream && l == 2;
           const uint64_t wd = l == 1 ? whdesc[1] : whdesc[2];
+          // fp16/bf16: the layer's bias first (D = ones x bias-block^T initialises the
+          // accumulator; it needs no H, so it is issued before the first chunk wait)
+          constexpr uint32_t kAcc = PREC == 2 ? 0u : 1u;
+          if constexpr (PREC != 2)
+            if (issuer)
+              ptx::mma_cg2<PREC>(d, onesdesc, wd + (tc_wh_half_bytes(PREC) >> 4), idesc, 0);
           for (uint32_t kc = 0; kc < kChunks; ++kc) {
 #ifndef LAKE_ABL_NOHREADY  // timing-only ablation: the MMA never waits for H chunks
             ptx::mbar_wait(bar(B_HREADY + kc), (h_phase >> kc) & 1);
@@ -695,7 +719,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
                 if (issuer)
                   ptx::mma_cg2_ts<PREC>(d, ha + tmem_a_col<PREC>(ks),
                                       ringdesc + (slot * kTcRingSlotBytes >> 4) + (s % kSPS) * kStep,
-                                      idesc, ks);
+                                      idesc, ks | kAcc);
                 if (s % kSPS == kSPS - 1) {
                   if (issuer) ptx::mma_commit_cg2(bar(B_REMPTY + slot), 0x3);
                   ++mc;
@@ -706,7 +730,8 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
               for (uint32_t s = 0; s < kKS; ++s) {
                 const uint32_t ks = kc * kKS + s;
                 if (issuer)
-                  ptx::mma_cg2_ts<PREC>(d, ha + tmem_a_col<PREC>(ks), wd + ks * kStep, idesc, ks);
+                  ptx::mma_cg2_ts<PREC>(d, ha + tmem_a_col<PREC>(ks), wd + ks * kStep, idesc,
+                                        ks | kAcc);
               }
             }
             __syncwarp();
@@ -971,7 +996,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
 // chunk loop small - two variants cost ~40% more instructions and I-cache misses)
 #define EPI_H(R) epi_to_h_tmem<PREC, W>(R, hbias + l * kHidden, col0, tbase)
 // (NN: the staged last-layer bias is b0, zeroed at staging because the MMA added it)
-#define EPI_L(R) epi_to_logits<W>(R, bl, wo, col0, p)
+#define EPI_L(R) epi_to_logits<PREC, W>(R, bl, wo, col0, p)
         ptx::tmem_ld_cols<W>(tbase + col_of(0), ra);
         ptx::tmem_ld_wait();
         if (!last) {
