@@ -1,21 +1,15 @@
 #!/bin/bash
-# Evidence for profiles/: ncu launch list of the default bench command and one ncu --set full
-# capture of the dominant kernel (fused tcgen05 MLP), plus the digitise kernel at C5 size.
+# round profiles: full GPU suite, smoke, default bench line, ncu launch list + full capture of
+# the fused kernel (C5), report mode
 mkdir -p gpurun_out
-TAG=${1:-r1}
-timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv \
-    --log-file gpurun_out/launches_$TAG.csv python bench.py --steps 3 --warmup 3 --no-e2e --no-cpu \
-    > gpurun_out/launches_$TAG.out 2>&1
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:mlp_tc_kernel -s 3 -c 1 \
-    -o gpurun_out/full_tc_$TAG python bench.py --steps 1 --warmup 3 --no-e2e --no-cpu \
-    > gpurun_out/full_tc_$TAG.out 2>&1
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:mlp_fp32_kernel -s 1 -c 1 \
-    -o gpurun_out/full_fp32_$TAG python bench.py --config C3 --prec fp32 --steps 1 --warmup 1 --no-e2e --no-cpu \
-    > gpurun_out/full_fp32_$TAG.out 2>&1
-timeout 300 ncu --set full --clock-control none -k regex:digitize_kernel -c 1 \
-    -o gpurun_out/full_dig_$TAG python scripts/run_digitize.py > gpurun_out/full_dig_$TAG.out 2>&1
-for m in mllb kml; do
-  timeout 300 ncu --set full --clock-control none --import-source on -k regex:mlp_family -s 1 -c 1 \
-      -o gpurun_out/full_fam${m}_$TAG python scripts/run_family.py $m > gpurun_out/full_fam${m}_$TAG.out 2>&1
-done
-echo done
+timeout 1500 python -m pytest tests -m gpu -q -rf -p no:cacheprovider > gpurun_out/t_all.log 2>&1
+echo "exit $?" >> gpurun_out/t_all.log
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1
+echo "exit $?" >> gpurun_out/smoke.log
+timeout 600 python bench.py > gpurun_out/bench_default.json 2> gpurun_out/bench_default.err
+timeout 300 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none -c 60 --csv \
+    --log-file gpurun_out/launches_r2.csv python bench.py --steps 3 --warmup 1 --no-e2e --no-cpu --no-latency > gpurun_out/launches_r2.out 2>&1
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:mlp_tc -s 1 -c 1 \
+    -o gpurun_out/prof_r2_tc python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu --no-latency > gpurun_out/prof_r2_tc.out 2>&1
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:group_scatter -s 1 -c 1 \
+    -o gpurun_out/prof_r2_scatter python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu --no-latency > gpurun_out/prof_r2_scatter.out 2>&1

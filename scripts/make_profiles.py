@@ -42,7 +42,7 @@ if os.path.exists(lpath):
     tot = sum(sum(v) for v in per.values())
     with open(os.path.join(out, f"{tag}_launches.txt"), "w") as f:
         f.write(f"# ncu --metrics gpu__time_duration.sum --clock-control none, command: "
-                f"python bench.py --steps 3 --warmup 3 --no-e2e --no-cpu (C5, tcgen05 f16)\n")
+                f"python bench.py --steps 3 --warmup 1 --no-e2e --no-cpu --no-latency (C5, tcgen05 f16)\n")
         f.write("# kernel, launches, total us, mean us, share of all launched time\n")
         for name, v in sorted(per.items(), key=lambda x: -sum(x[1])):
             f.write(f"{name:40s} {len(v):4d} {sum(v):12.1f} {sum(v)/len(v):10.1f} {100*sum(v)/tot:6.2f}%\n")
@@ -63,7 +63,7 @@ KEYS = ["gpu__time_duration.sum", "sm__cycles_elapsed.avg.per_second",
         "launch__shared_mem_per_block_dynamic", "sm__warps_active.avg.pct_of_peak_sustained_active",
         "smsp__issue_active.avg.pct_of_peak_sustained_active"]
 for kind, key in (("tc", "C5_f16_g1"), ("fp32", "C3_fp32_g1"), ("dig", None),
-                  ("fammllb", "FAM_mllb_g1"), ("famkml", "FAM_kml_g1")):
+                  ("fammllb", "FAM_mllb_g1"), ("famkml", "FAM_kml_g1"), ("scatter", None)):
     rep = os.path.join(src, f"full_{kind}_{tag}.ncu-rep")
     if not os.path.exists(rep):
         continue
