@@ -96,7 +96,9 @@ enum lake_arch {
  * DESIGN.md §7): 64 per-SSD models fit in one byte. An id the type cannot hold a loaded model
  * for is simply unknown (decision 0, NaN logits). */
 enum lake_flags {
-    LAKE_IN_DIGITS  = 0x00, /* in = const uint8_t[n][32] (pad byte must be 0)           */
+    LAKE_IN_DIGITS  = 0x00, /* in = const uint8_t[n][32]: digits 0..9 (bytes 0..30; the
+                               tensor-core multi-model path packs them into 4-bit fields)
+                               and a pad byte that is ignored                              */
     LAKE_IN_RAW     = 0x01, /* in = const lake_io_raw_t[n]; digitised inside the kernel  */
     LAKE_PREC_FP32  = 0x00, /* CUDA-core FP32, strict operation order: bit-exact with the
                                oracle (DESIGN.md §3 reading R15)                           */
@@ -165,7 +167,10 @@ int lake_linnos_digitize(const lake_io_raw_t *raw, int64_t n, uint8_t *digits, v
  *   decisions : device uint8_t[n]; 1 = slow, 0 = fast. decision = logit[1] > logit[0]
  *               (ties and NaN -> 0).
  *   logits    : device float[n][2] or NULL (not written).
- * Fused: digitise (RAW input) -> every layer -> argmax in one kernel. */
+ * Fused: digitise (RAW input) -> every layer -> argmax in one kernel. Tensor-core paths
+ * bulk-copy each tile's contiguous input rows (16-B aligned input; otherwise per-row loads).
+ * FP32 with n <= 64 (NN: <= 8) runs on one 8-CTA cluster (same strict-order arithmetic).
+ * Never allocates; capturable in a CUDA graph. */
 int lake_linnos_infer(const void *in, uint32_t flags, int64_t n, int32_t model_id,
                       uint8_t *decisions, float *logits, void *stream);
 
@@ -176,7 +181,8 @@ size_t lake_linnos_workspace_bytes(int64_t n);
  * device): I/O i is scored with model model_ids[i] (device array of n elements
  * of the type flags & LAKE_IDS_MASK selects: int32_t by default, uint16_t, uint8_t).
  * Groups I/Os by model on the device (histogram, scan, scatter of indices; the order inside
- * a model's group is not preserved and does not affect any result), then
+ * a model's group is not preserved and does not affect any result; tensor-core paths also
+ * write each I/O's digits as a 16-byte packed row at its grouped position), then
  * runs the fused kernel over model-homogeneous tiles and scatters results back to the
  * caller's order. Results equal per-model lake_linnos_infer calls bit for bit.
  * workspace: device buffer of at least lake_linnos_workspace_bytes(n) bytes (else
