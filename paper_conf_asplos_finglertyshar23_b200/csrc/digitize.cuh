@@ -68,13 +68,63 @@ __device__ __forceinline__ uint4 pack_slots(const uint32_t (&dg)[32] /* canonica
   return make_uint4(w[0], w[1], w[2], w[3]);
 }
 
-// Packed row of one raw record.
-__device__ __forceinline__ uint4 pack_record(const uint32_t (&rec)[9]) {
+// Packed row of one raw record, reference form (digit by digit through pack_slots).
+__device__ __forceinline__ uint4 pack_record_digits(const uint32_t (&rec)[9]) {
   uint32_t dg[32];
 #pragma unroll
   for (int i = 0; i < 32; ++i) dg[i] = 0;
   digitize_record(rec, [&](int k, uint32_t v) { dg[k] = v; });
   return pack_slots(dg);
+}
+
+// SWAR digit pairs: for two values a, b < 100 held as x = a | b << 16, returns
+// p(a) | p(b) << 16 with p(y) = (y / 10) | (y % 10) << 4, the packed byte of a two-digit
+// field (tens in slot 2p, ones in slot 2p+1). y / 10 = (y * 205) >> 11 for y < 1029; the
+// halves cannot carry into each other (y * 205 < 2^15), and p(y) = 16 y - 159 (y / 10).
+__host__ __device__ __forceinline__ uint32_t bcd_pair2(uint32_t x) {
+  const uint32_t t = ((x * 205u) >> 11) & 0x000F000Fu;
+  return 16u * x - 159u * t;
+}
+// Hundreds split of two values a, b <= 999 held as x = a | b << 16: hi = v / 100 per half
+// ((v * 41) >> 12 for v <= 999: checked exhaustively by tests/test_pack_swar.py), lo = v - 100 hi.
+__host__ __device__ __forceinline__ uint32_t hundreds_pair3(uint32_t x) {
+  return ((x * 41u) >> 12) & 0x000F000Fu;
+}
+
+// Packed row of one raw record (same bytes as pack_record_digits; ~90 integer ops instead of
+// ~230: the grouping pass that writes these rows was ALU-issue bound on the digit-by-digit
+// form). Layout (tc_slot_digit): bytes 0-7 = p(lat_f / 100), p(lat_f % 100) for f = 0..3;
+// bytes 8-12 = p(q % 100) for q_now, q_hist[0..3]; bytes 13-15 = the five leading queue
+// digits paired low-nibble first, then the constant 1 of slot 31.
+__host__ __device__ __forceinline__ uint4 pack_record(const uint32_t (&rec)[9]) {
+  uint32_t w01[2];
+#pragma unroll
+  for (int k = 0; k < 2; ++k) {  // two latency fields per word
+    uint32_t half[2];
+#pragma unroll
+    for (int j = 0; j < 2; ++j) {
+      const uint32_t v = rec[1 + 2 * k + j] < 9999u ? rec[1 + 2 * k + j] : 9999u;
+      const uint32_t hi = (v * 5243u) >> 19;  // v / 100 for v < 43699
+      const uint32_t p = bcd_pair2(hi | (v - 100u * hi) << 16);
+      half[j] = (p & 0xFFu) | ((p >> 8) & 0xFF00u);
+    }
+    w01[k] = half[0] | half[1] << 16;
+  }
+  uint32_t q[5];
+#pragma unroll
+  for (int g = 0; g < 5; ++g) {
+    const uint32_t r = g == 0 ? rec[0] : rec[4 + g];
+    q[g] = r < 999u ? r : 999u;
+  }
+  const uint32_t x01 = q[0] | q[1] << 16, x23 = q[2] | q[3] << 16;
+  const uint32_t h01 = hundreds_pair3(x01), h23 = hundreds_pair3(x23), h4 = (q[4] * 41u) >> 12;
+  const uint32_t p01 = bcd_pair2(x01 - 100u * h01), p23 = bcd_pair2(x23 - 100u * h23);
+  const uint32_t p4 = bcd_pair2(q[4] - 100u * h4);
+  const uint32_t w2 = (p01 & 0xFFu) | ((p01 >> 8) & 0xFF00u) | (p23 & 0xFFu) << 16 |
+                      ((p23 >> 16) & 0xFFu) << 24;
+  const uint32_t w3 = (p4 & 0xFFu) | (h01 & 0xFu) << 8 | (h01 >> 16) << 12 | (h23 & 0xFu) << 16 |
+                      (h23 >> 16) << 20 | h4 << 24 | 1u << 28;
+  return make_uint4(w01[0], w01[1], w2, w3);
 }
 
 // Packed row of a LAKE_IN_DIGITS row (bytes 0..30 are digits 0..9).
