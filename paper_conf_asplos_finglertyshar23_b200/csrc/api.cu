@@ -218,17 +218,28 @@ int current_model(int32_t model_id, int *device, DevModel *out, const DevModel *
   return LAKE_OK;
 }
 
-int current_table(int *device, const DevModel **table, int *any) {
+// *any: some model is loaded; *max_nh: the most hidden layers among the loaded models (the
+// tensor-core kernel's SMEM layout for a multi-model call; tiles of a model loaded after this
+// snapshot are clamped to it on the device, which keeps memory safe under that race).
+// *has_nn: some loaded model is an NN (one hidden layer).
+int current_table(int *device, const DevModel **table, int *any, int *max_nh = nullptr,
+                  int *has_nn = nullptr) {
   if (cudaGetDevice(device) != cudaSuccess) return LAKE_ERR_CUDA;
   std::lock_guard<std::mutex> lk(g_mu);
   *any = 0;
+  if (max_nh) *max_nh = 1;
+  if (has_nn) *has_nn = 0;
   if (*device < 0 || *device >= kMaxDevices || !g_dev[*device] || !g_dev[*device]->init) {
     *table = nullptr;
     return LAKE_OK;
   }
   *table = g_dev[*device]->table;
   for (int i = 0; i < LAKE_MAX_MODELS; ++i)
-    if (g_dev[*device]->host[i].arch >= 0) { *any = 1; break; }
+    if (g_dev[*device]->host[i].arch >= 0) {
+      *any = 1;
+      if (max_nh && g_dev[*device]->host[i].nh > *max_nh) *max_nh = g_dev[*device]->host[i].nh;
+      if (has_nn && g_dev[*device]->host[i].nh == 1) *has_nn = 1;
+    }
   return LAKE_OK;
 }
 
@@ -576,9 +587,9 @@ int multi_grouped_impl(const void *in, uint32_t flags, int64_t n, uint8_t *decis
   if (!in || !decisions || !workspace) return LAKE_ERR_INVAL;
   if (check_input_ptr(in, in_kind) != LAKE_OK) return LAKE_ERR_INVAL;
   if (ws_bytes < group_workspace_bytes(n)) return LAKE_ERR_NOMEM;
-  int device, any;
+  int device, any, max_nh, has_nn;
   const DevModel *table;
-  rc = current_table(&device, &table, &any);
+  rc = current_table(&device, &table, &any, &max_nh, &has_nn);
   if (rc != LAKE_OK) return rc;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   cudaError_t e = launch_unknown_fill(workspace, n, decisions, logits, s);
@@ -591,7 +602,15 @@ int multi_grouped_impl(const void *in, uint32_t flags, int64_t n, uint8_t *decis
   TileSched ts;
   std::memset(&ts, 0, sizeof(ts));
   group_sched(workspace, n, prec < 0 ? 0 : 1, table, &ts);
-  return launch_main(in, in_kind, prec, ts, 3, decisions, logits, s, device);
+  if ((prec == 0 || prec == 1) && has_nn && max_nh > 1) {
+    // NN and NN+1/NN+2 models loaded: the grouping put the NN tiles first; one kernel per
+    // class (the NN kernel runs the output layer on the tensor cores, mlp_tc.cu)
+    ts.part = 1;
+    rc = launch_main(in, in_kind, prec, ts, 1, decisions, logits, s, device);
+    if (rc != LAKE_OK) return rc;
+    ts.part = 2;
+  }
+  return launch_main(in, in_kind, prec, ts, max_nh, decisions, logits, s, device);
 }
 
 int lake_linnos_infer_multi(const void *in, uint32_t flags, int64_t n, const int32_t *model_ids,

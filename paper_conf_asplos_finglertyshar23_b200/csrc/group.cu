@@ -34,9 +34,11 @@ struct WsHeader {
   int32_t cursor_unused[LAKE_MAX_MODELS];  // (cursors live in WsLayout::cursor, padded)
   int32_t offsets[LAKE_MAX_MODELS];
   int32_t tile_off64[LAKE_MAX_MODELS + 1];
-  int32_t tile_off256[LAKE_MAX_MODELS + 1];
+  int32_t tile_off256[LAKE_MAX_MODELS + 1];  // by rank in ord256 (NN models first)
+  int32_t ord256[LAKE_MAX_MODELS];           // rank -> model slot
   int32_t n_tiles64;
   int32_t n_tiles256;
+  int32_t n_tiles256_nn;                     // the NN models' tiles: [0, n_tiles256_nn)
   int32_t n_known;
   int32_t unk_cursor;
   int64_t n_unknown;
@@ -47,6 +49,7 @@ struct WsHeader {
   // (not used by this call's known models) meanwhile; a divergent view would overrun a
   // model's reserved range of perm
   uint8_t known[LAKE_MAX_MODELS];
+  uint8_t nnc[LAKE_MAX_MODELS];  // ... and holds an NN model (one hidden layer), same snapshot
 };
 
 __host__ __device__ inline size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
@@ -116,6 +119,7 @@ group_init(const DevModel *__restrict__ table, WsHeader *h) {
   uint32_t *w = reinterpret_cast<uint32_t *>(h);
   for (uint32_t i = threadIdx.x; i < offsetof(WsHeader, known) / 4; i += blockDim.x) w[i] = 0;
   h->known[threadIdx.x] = table[threadIdx.x].arch >= 0 ? 1 : 0;
+  h->nnc[threadIdx.x] = (table[threadIdx.x].arch >= 0 && table[threadIdx.x].nh == 1) ? 1 : 0;
 }
 __device__ __forceinline__ int32_t bin_of(const uint8_t *known_s, int32_t m) {
   return ((unsigned)m < (unsigned)LAKE_MAX_MODELS && known_s[m]) ? m : LAKE_MAX_MODELS;
@@ -194,15 +198,27 @@ group_scan(WsHeader *h, int32_t *cursor) {
   const int32_t t64 = block_excl_scan((c + kF32TileM - 1) / kF32TileM, warp_tot, &total);
   h->tile_off64[m] = t64;
   const int32_t tot64 = total;
-  const int32_t t256 = block_excl_scan((c + kTcTileRows - 1) / kTcTileRows, warp_tot, &total);
-  h->tile_off256[m] = t256;
+  // tensor-core tiles: NN models' first (slot order within each class), so that the NN tiles
+  // form the prefix [0, n_tiles256_nn) that the NN kernel takes (api.cu: multi-model calls
+  // mixing NN with NN+1/NN+2 run one kernel per class)
+  const bool nn = h->nnc[m] != 0;
+  const int32_t tc = (c + kTcTileRows - 1) / kTcTileRows;
+  const int32_t t_nn = block_excl_scan(nn ? tc : 0, warp_tot, &total);
+  const int32_t tot_nn = total;
+  const int32_t t_ot = block_excl_scan(nn ? 0 : tc, warp_tot, &total);
+  const int32_t tot256 = tot_nn + total;
+  const int32_t r_nn = block_excl_scan(nn ? 1 : 0, warp_tot, &total);
+  const int32_t rank = nn ? r_nn : total + (m - r_nn);
+  h->ord256[rank] = m;
+  h->tile_off256[rank] = nn ? t_nn : tot_nn + t_ot;
   if (m == 0) {
     h->n_known = n_known;
     cursor[LAKE_MAX_MODELS * kCursorStride] = n_known;
     h->n_tiles64 = tot64;
-    h->n_tiles256 = total;
+    h->n_tiles256 = tot256;
+    h->n_tiles256_nn = tot_nn;
     h->tile_off64[LAKE_MAX_MODELS] = tot64;
-    h->tile_off256[LAKE_MAX_MODELS] = total;
+    h->tile_off256[LAKE_MAX_MODELS] = tot256;
   }
 }
 
@@ -429,8 +445,9 @@ __global__ void group_tiles(const WsHeader *__restrict__ h, int64_t max64, int64
     t64_count[t] = rem < kF32TileM ? rem : kF32TileM;
   }
   if (t < h->n_tiles256 && t < max256) {
-    const int m = find_model(h->tile_off256, (int32_t)t);
-    const int32_t local = (int32_t)t - h->tile_off256[m];
+    const int k = find_model(h->tile_off256, (int32_t)t);
+    const int m = h->ord256[k];
+    const int32_t local = (int32_t)t - h->tile_off256[k];
     const int32_t rem = h->counts[m] - local * kTcTileRows;
     t256_model[t] = m;
     t256_begin[t] = (int64_t)h->offsets[m] + (int64_t)local * kTcTileRows;
@@ -479,6 +496,7 @@ struct GroupPtrs {
   int64_t *tb[2];
   int32_t *tc[2];
   int32_t *nt[2];
+  int32_t *split;  // NN-class prefix of the 256-row tile list
   int64_t max[2];
   int32_t *cc;  // per-chunk histograms
   uint4 *pdig;  // packed digit rows, grouped order
@@ -502,6 +520,7 @@ static GroupPtrs group_ptrs(void *ws, int64_t n) {
   p.cursor = reinterpret_cast<int32_t *>(b + L.cursor);
   p.nt[0] = &p.h->n_tiles64;
   p.nt[1] = &p.h->n_tiles256;
+  p.split = &p.h->n_tiles256_nn;
   p.max[0] = L.max64;
   p.max[1] = L.max256;
   return p;
@@ -572,6 +591,7 @@ cudaError_t launch_group_pack(void *ws, int64_t n, const void *in, int in_kind, 
 
 void group_sched(void *ws, int64_t n, int which, const DevModel *table, TileSched *ts) {
   GroupPtrs p = group_ptrs(ws, n);
+  ts->tile_split_dev = which == 1 ? p.split : nullptr;
   ts->pdig = which == 1 ? p.pdig : nullptr;
   ts->tile_model = p.tm[which];
   ts->tile_begin = p.tb[which];

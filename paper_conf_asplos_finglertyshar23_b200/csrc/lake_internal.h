@@ -127,6 +127,9 @@ struct TileSched {
   int64_t n;                   // I/Os
   const DevModel *table;       // device model table (multi)
   DevModel model;              // single-model copy
+  int nh_cap;                  // tcgen05 path: the SMEM layout's hidden-layer count (set at launch)
+  const int32_t *tile_split_dev;  // multi (tcgen05): NN tiles are [0, *split), the rest after
+  int part;                    // 0: every tile; 1: tiles [0, *split); 2: tiles [*split, n_tiles)
 };
 
 // Kernel launchers (return cudaError_t of the launch).

@@ -88,7 +88,8 @@ __device__ unsigned long long *g_lake_trace = nullptr;
 enum TraceKind { T_XFULL = 1, T_TEMPTY = 2, T_HREADY = 3, T_COMMIT = 4, T_DFULL = 5,
                  T_CHUNK = 6, T_LAYER_END = 7, T_XEMPTY = 8, T_XARRIVE = 9, T_ISSUED = 10,
                  T_LDWAIT = 11, T_STS = 12, T_FENCE = 13, T_TOP = 14, T_SCHED = 15,
-                 T_WREADY = 16, T_MMA0 = 17, T_CX = 18 };
+                 T_WREADY = 16, T_MMA0 = 17, T_CX = 18, T_OHDONE = 19, T_OCOMMIT = 20,
+                 T_EHDONE = 21, T_EDOUT = 22, T_ETEMPTY = 23 };
 
 // H (the next layer's A operand) stays in tensor memory, packed in place into the
 // accumulator it came from (default); -DLAKE_H_SMEM restores the SMEM H tile + proxy fences.
@@ -161,11 +162,39 @@ __host__ __device__ constexpr bool streams_w2(int nh, int prec) {
 __host__ __device__ constexpr uint32_t kStageBytes(int prec) { return prec == 2 ? 2048u : 4608u; }
 
 struct Layout {
-  uint32_t ring, h, x, stage, t100, ones, prm, red, prm0, red0, bar, total;
+  uint32_t ring, h, x, stage, t100, ones, prm, red, prm0, red0, wout, bar, total;
 };
+// NN kernels (layout 1) with fp16/bf16 operands (out_on_tc): the 2-wide output layer runs on
+// the tensor cores. The draining epilogue group packs ReLU(H) in place into the accumulator
+// (as for a hidden layer), the MMA issuer multiplies it (A from TMEM) by W_out (N = 16, rows
+// 2..15 zero) into the accumulator's last 16 columns, and the group reads back two of them.
+// To free those 16 columns the last K-step's packed H goes into the unused half of K-step 13's
+// (same warp, earlier chunk: program order makes the overwrite safe). NN tiles were bound by
+// the epilogue's CUDA-core work (ReLU + 512 FMAs per row); this leaves 128 packed conversions
+// per row. (An SMEM A tile was 3x slower: N=16 SS MMAs ran at ~90 cycles each.) Every
+// fp16/bf16 NN tile runs in such a kernel (multi-model calls that mix NN with NN+1/NN+2 run
+// one kernel per class, api.cu), so an NN tile gives the same bits in a single-model call and
+// inside any multi-model call, and the NN+1/NN+2 kernels carry none of this code.
+#ifndef LAKE_NO_OTC
+__host__ __device__ constexpr bool out_on_tc(int nh_layout, int prec) {
+  return kEpiGroups == 2 && nh_layout == 1 && prec != 2;
+}
+#else  // A/B switch: output layer on CUDA cores for NN too
+__host__ __device__ constexpr bool out_on_tc(int, int) { return false; }
+#endif
+constexpr uint32_t kWoutBytes = 8u * kHidden * 2;    // one group's W_out block (8 rows x K 256)
+constexpr uint32_t kLboR8 = 8 * 16;                  // K-direction core stride, 8-row operand
+constexpr uint32_t kOutDCol = kHidden - 16;          // output accumulator: columns 240..255
+constexpr uint32_t kOutLastA = 13 * 16 + 8;          // last K-step's packed H: K-step 13's gap
+__host__ __device__ constexpr uint32_t otc_wout(int prec) { return tc_w0_half_bytes(prec); }
+__host__ __device__ constexpr uint32_t otc_end(int prec) { return otc_wout(prec) + 2 * kWoutBytes; }
+
 __host__ __device__ constexpr Layout tc_layout(int nh_layout, int prec) {
   Layout L{};
-  L.ring = align1k(tc_resident_bytes(nh_layout, prec));
+  // NN layout with the output layer on the tensor cores: the W_out blocks after W0
+  const uint32_t region = out_on_tc(nh_layout, prec) ? otc_end(prec)
+                                                      : tc_resident_bytes(nh_layout, prec);
+  L.ring = align1k(region);
   L.h = L.ring + (streams_w2(nh_layout, prec) ? kTcRingSlots * kTcRingSlotBytes : 0u);
   L.x = L.h + kHBytes;
   L.stage = L.x + 2 * x_bytes(prec);
@@ -177,8 +206,9 @@ __host__ __device__ constexpr Layout tc_layout(int nh_layout, int prec) {
   // groups, NN tiles (a single layer) are drained by the group of their accumulator buffer
   L.prm0 = L.red + kRedBytes;
   L.red0 = L.prm0 + kPrmFloats * 4;
+  L.wout = otc_wout(prec);  // behind W0 in the weight region (out_on_tc layouts only)
   L.bar = L.red0 + kRedBytes;
-  L.total = L.bar + 256;
+  L.total = L.bar + 512;
   return L;
 }
 static_assert(tc_layout(3, 2).total <= 232448, "tf32 NN+2 layout exceeds 227 KB");
@@ -191,10 +221,12 @@ enum : uint32_t {
   B_RFULL = 13 + kChunks,                 // [kTcRingSlots] W2 ring slot loaded (tf32 NN+2)
   B_REMPTY = B_RFULL + kTcRingSlots,      // [kTcRingSlots] W2 ring slot consumed
   B_SFULL = B_REMPTY + kTcRingSlots,     // [2] input staging buffer loaded (bulk copy)
-  B_COUNT = B_SFULL + 2
+  B_HDONE = B_SFULL + 2,                  // [2] out_on_tc: H of buffer b packed (both CTAs)
+  B_DOUT = B_HDONE + 2,                   // [2] out_on_tc: output MMA of buffer b done
+  B_COUNT = B_DOUT + 2
 };
 constexpr uint32_t kTmemSlot = B_COUNT * 8;  // u32 TMEM base address
-static_assert(kTmemSlot + 4 <= 256, "barrier block");
+static_assert(kTmemSlot + 4 <= 512, "barrier block");
 
 // Per-tile schedule entry. Each role loads tile t+1's entry at the top of tile t (the
 // global loads then overlap tile t's work instead of stalling the next iteration).
@@ -220,7 +252,9 @@ __device__ __forceinline__ TileInfo tile_info(const TileSched &ts, int64_t t) {
     ti.count = (int)(rem < kTcTileRows ? rem : kTcTileRows);
   }
   ti.img = ti.model->tc_img[PREC];
-  ti.nh = ti.model->nh;
+  // a model loaded after the host sized the layout (racing the call) is clamped to it: wrong
+  // logits for that model, but every role agrees and nothing outside the layout is touched
+  ti.nh = ti.model->nh < ts.nh_cap ? ti.model->nh : ts.nh_cap;
   return ti;
 }
 
@@ -427,7 +461,7 @@ __device__ __forceinline__ void epi_to_logits(const uint32_t (&r)[W], const floa
   }
 }
 
-template <int PREC, int IN_KIND>
+template <int PREC, int IN_KIND, bool OTC>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
 mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts, int nh_layout,
               uint8_t *__restrict__ decisions, float *__restrict__ logits) {
@@ -475,8 +509,14 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
 #endif
 #endif
   const int64_t n_tiles = ts.n_tiles_dev ? (int64_t)*ts.n_tiles_dev : ts.n_tiles;
-  const int64_t t_begin = n_tiles * cid / ncl;
-  const int64_t t_end = n_tiles * (cid + 1) / ncl;
+  int64_t t_lo = 0, t_hi = n_tiles;  // part 1 / 2: the NN-class prefix / the rest (multi)
+  if (ts.part) {
+    const int64_t sp = *ts.tile_split_dev < n_tiles ? (int64_t)*ts.tile_split_dev : n_tiles;
+    if (ts.part == 1) t_hi = sp;
+    else t_lo = sp;
+  }
+  const int64_t t_begin = t_lo + (t_hi - t_lo) * cid / ncl;
+  const int64_t t_end = t_lo + (t_hi - t_lo) * (cid + 1) / ncl;
 
   if (threadIdx.x == 0) {
     ptx::mbar_init(bar(B_WLOAD), 1);
@@ -497,6 +537,10 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       ptx::mbar_init(bar(B_REMPTY + i), 1);      // tcgen05.commit (multicast)
     }
     for (int i = 0; i < 2; ++i) ptx::mbar_init(bar(B_SFULL + i), 1);  // expect_tx arrive
+    for (int i = 0; i < 2; ++i) {
+      ptx::mbar_init(bar(B_HDONE + i), 2 * kGroupWarps);  // the draining group, both CTAs
+      ptx::mbar_init(bar(B_DOUT + i), 1);                 // tcgen05.commit (multicast)
+    }
     ptx::fence_mbar_init();
   }
   if (warp == kWarpLoad) {
@@ -644,7 +688,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           const DevModel *mm = slot_n >= 0 ? &ts.table[slot_n] : &ts.model;
           nxt.model = mm;
           nxt.img = mm->tc_img[PREC];
-          nxt.nh = mm->nh;
+          nxt.nh = mm->nh < ts.nh_cap ? mm->nh : ts.nh_cap;
         }
         slot_n = slot_nn;
         LAKE_TEV(T_SCHED, it, 0, 0);
@@ -654,7 +698,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           cur = ti.img;
         }
         LAKE_TEV(T_WREADY, it, 0, 0);
-        const int nh = ti.nh;
+        const int nh = OTC ? 1 : ti.nh;  // an out_on_tc kernel only runs NN tiles
         const bool stream = streams_w2(nh, PREC);
         const uint32_t xb = (uint32_t)(it & 1);
         {  // layer 0: D = X[128(x2) x 32] * W0^T
@@ -743,8 +787,8 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           LAKE_TEV(T_COMMIT, it, l, 0);
           ++g;
         }
-        if (t + 1 < t_end && nxt.img != cur && issuer)
-          ptx::mma_commit_cg2(bar(B_WFREE), 0x3);  // old weights no longer read
+        const bool wswitch = t + 1 < t_end && nxt.img != cur;
+        if (wswitch && issuer) ptx::mma_commit_cg2(bar(B_WFREE), 0x3);  // old weights no longer read
         __syncwarp();
       }
     }
@@ -814,6 +858,11 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         for (int half = 0; half < 2; ++half) {
           const uint32_t r = d + 64 * half;
           const bool valid = r < rows;
+#ifdef LAKE_ABL_NODIG  // timing-only ablation: no digitiser conversion (staged inputs)
+#pragma unroll
+          for (int i = 0; i < (PREC == 2 ? 32 : 16); ++i) xr[half].w[i] = r + i + st[0];
+          if (true) continue;
+#endif
           if (ts.pdig) {
             row_from_packed<PREC>(valid ? *reinterpret_cast<const uint4 *>(st + r * 16)
                                         : make_uint4(0, 0, 0, 0), xr[half]);
@@ -931,6 +980,9 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
     const bool do_last = kEpiGroups == 1 || gy == 1;  // converts the last layer
     const uint32_t hready_leader0 = ptx::mapa(bar(B_HREADY), 0);
     const uint32_t tempty_leader0 = ptx::mapa(bar(B_TEMPTY), 0);
+    uint32_t do_phase = 0, hd_phase = 0;  // out_on_tc: B_DOUT / B_HDONE phases per buffer
+    const uint32_t hdone_leader0 = ptx::mapa(bar(B_HDONE), 0);
+    const DevModel *wcur = nullptr;  // out_on_tc: model of this group's W_out block
     const bool own0 = kEpiGroups == 2 && gy == 0;  // group 0's private output-layer copy
     float *prm = reinterpret_cast<float *>(smem + (own0 ? L.prm0 : L.prm));  // last b | W_out | b_out
     float *hbias = reinterpret_cast<float *>(smem + L.prm + kPrmFloats * 4);  // H-layer biases
@@ -944,7 +996,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
     for (int64_t t = t_begin; t < t_end; ++t, ++it) {
       const TileInfo ti = nxt;
       if (t + 1 < t_end) nxt = tile_info<PREC>(ts, t + 1);
-      const int nh = ti.nh;
+      const int nh = OTC ? 1 : ti.nh;  // an out_on_tc kernel only runs NN tiles
       if (ti.model != cur) {
         // stage this model's epilogue parameters (each group the ones it uses): fp32 biases
         // of the H layers, fp32 last-layer bias | W_out | b_out
@@ -1033,6 +1085,105 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
             if (kPrefetch && j + 1 < kWarpChunks) ptx::tmem_ld_wait();
             LAKE_TEV(T_LDWAIT, it, l, kc);
           }
+        } else if (OTC) {  // (every tile of an out_on_tc kernel is an NN tile)
+          // NN, output layer on the tensor cores: H -> ReLU -> fp16/bf16, packed in place (the
+          // A operand of the output MMA, as for a hidden layer); then this group's leader-CTA
+          // poller issues the output layer once the whole group (both CTAs) has packed H. An
+          // M=256 MMA costs >= 64 cycles whatever its N (scripts/microbench/umma_rate.cu), so
+          // the 16 N=16 K-steps take ~1k tensor cycles; issued by the layer-0 thread they
+          // blocked it that long, here they queue while layer 0 of later tiles goes on. Buffer
+          // reuse stays ordered by TEMPTY: the group releases the accumulator only after
+          // reading the result (DOUT). (Issuing the K-steps chunk by chunk as the packing
+          // progresses measured 30% slower: per-chunk group barriers on the packing path.)
+          const int pos = (int)(rank * 128 + row);
+          const int64_t pp = ti.begin + pos;
+          const int64_t io = (ts.perm && pos < ti.count) ? (int64_t)__ldg(ts.perm + pp) : pp;
+          static_assert(kEpiCols == 16 && kChunks == 8 && kEpiPerQ == 2, "OTC packing layout");
+          if (ti.model != wcur) {
+            // this group's W_out block, rewritten whole (the region held another model's
+            // weights in between): leader CTA rows 0, 1 = W_out, zeros elsewhere. Safe here:
+            // the accumulator is full, so this model's weights are resident and every MMA of
+            // an earlier model (and this group's previous output MMA) has completed.
+            const float *wsrc = ti.model->b[0] + kHidden;  // NN: b0 | W_out[2][256] | b_out
+            uint32_t *wblk = reinterpret_cast<uint32_t *>(smem + L.wout + gy * kWoutBytes);
+            for (uint32_t i = et; i < kWoutBytes / 4; i += NG) {
+              // word i: core column kc = i / 32, row r = (i / 4) % 8, k = 8 kc + 2 (i % 4)
+              const uint32_t r = (i >> 2) & 7u, k = (i >> 5) * 8 + 2 * (i & 3u);
+              uint32_t v = 0;
+              if (rank == 0 && r < 2) {
+                const float w0 = __ldg(wsrc + r * kHidden + k), w1 = __ldg(wsrc + r * kHidden + k + 1);
+                v = PREC == 0 ? (uint32_t)__half_as_ushort(__float2half_rn(w0)) |
+                                    ((uint32_t)__half_as_ushort(__float2half_rn(w1)) << 16)
+                              : (uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(w0)) |
+                                    ((uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(w1)) << 16);
+              }
+              wblk[i] = v;
+            }
+            ptx::fence_proxy_async_smem();  // read by the output MMA (after the HDONE arrive)
+            wcur = ti.model;
+          }
+#pragma unroll kEpiUnroll
+          for (uint32_t j = 0; j < kWarpChunks; ++j) {
+            const uint32_t col0 = col_of(j);
+            if (j + 1 < kWarpChunks) {
+              if (j & 1) ptx::tmem_ld_cols<W>(tbase + col_of(j + 1), ra);
+              else ptx::tmem_ld_cols<W>(tbase + col_of(j + 1), rb);
+            }
+            // the last K-step (chunk 7, second half) lands in K-step 13's free half, which
+            // this warp read in chunk 6; columns 240..255 stay free for the output MMA
+            const uint32_t dst = (j == kWarpChunks - 1 && hh == 1) ? kOutLastA : col0;
+            if (j & 1) epi_to_h_tmem<PREC, W>(rb, hbias, dst, tbase);
+            else epi_to_h_tmem<PREC, W>(ra, hbias, dst, tbase);
+            if (j + 1 < kWarpChunks) ptx::tmem_ld_wait();
+          }
+          ptx::tmem_st_wait();
+          ptx::tc_fence_before();
+          __syncwarp();
+          if (lane == 0) ptx::mbar_arrive_cluster(hdone_leader0 + b * 8);
+          LAKE_TEV(T_EHDONE, it, b, warp);
+          if (rank == 0 && lw == 1) {
+            ptx::mbar_wait(bar(B_HDONE + b), (hd_phase >> b) & 1);
+            ptx::tc_fence_after();
+            const bool issuer = lane == 0;
+            const uint32_t tm = __shfl_sync(0xffffffffu, tmem, 0);
+            const uint32_t idesc_out = ptx::umma_idesc_f16(PREC, 256, 16);
+            // this group's W_out block; A = the packed H in place (K-step 15 moved: kOutLastA)
+            const uint64_t wd = ptx::umma_desc(sbase + L.wout + gy * kWoutBytes, kLboR8, 1024);
+            const uint32_t acc = tm + b * 256;
+#pragma unroll
+            for (uint32_t ks = 0; ks < kHidden / 16; ++ks)
+              if (issuer)
+                ptx::mma_cg2_ts<PREC>(acc + kOutDCol,
+                                      acc + (ks + 1 == kHidden / 16 ? kOutLastA : tmem_a_col<PREC>(ks)),
+                                      wd + ks * ((2 * kLboR8) >> 4), idesc_out, ks);
+            if (issuer) ptx::mma_commit_cg2(bar(B_DOUT + b), 0x3);
+            __syncwarp();
+            LAKE_TEV(T_OCOMMIT, it, b, 0);
+          }
+          hd_phase ^= (1u << b);
+          if (lw == 1) ptx::mbar_wait(bar(B_DOUT + b), (do_phase >> b) & 1);
+          ptx::named_bar_sync(2 + gy, NG);
+          LAKE_TEV(T_EDOUT, it, b, warp);
+          do_phase ^= (1u << b);
+          ptx::tc_fence_after();
+          uint32_t o[2] = {0u, 0u};
+          if (hh == 0) {
+            ptx::tmem_ld_32x32b_x2(tbase + kOutDCol, o);
+            ptx::tmem_ld_wait();
+          }
+          ptx::tc_fence_before();
+          __syncwarp();
+          if (lane == 0) ptx::mbar_arrive_cluster(tempty_leader0 + b * 8);
+          LAKE_TEV(T_ETEMPTY, it, b, warp);
+          if (hh == 0 && pos < ti.count) {
+            const float l0 = __uint_as_float(o[0]) + wo[2 * kHidden + 0];
+            const float l1 = __uint_as_float(o[1]) + wo[2 * kHidden + 1];
+            if (logits) {
+              logits[io * 2 + 0] = l0;
+              logits[io * 2 + 1] = l1;
+            }
+            decisions[io] = (l1 > l0) ? 1 : 0;
+          }
         } else {
           // last hidden layer: fold the 2-neuron output layer (fp32, CUDA cores). The row's
           // output index is loaded first: with model-grouped staged inputs nothing else has
@@ -1061,7 +1212,6 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
               EPI_L(ra);
             }
           }
-#undef EPI_H
 #undef EPI_L
           // accumulator b fully read: release it before the reduction and the output stores
           ptx::tc_fence_before();
@@ -1097,6 +1247,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
             }
           }
         }
+#undef EPI_H
         if (!last) {  // accumulator b fully read by this warp (the last layer released it above)
           ptx::tc_fence_before();
           __syncwarp();
@@ -1133,42 +1284,46 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
 #endif
 }
 
-template <int PREC, int IN_KIND>
+template <int PREC, int IN_KIND, bool OTC>
 cudaError_t launch_t(const void *in, const TileSched &ts, int nh_layout, uint8_t *dec,
                      float *logits, cudaStream_t s, int grid) {
   const Layout L = tc_layout(nh_layout, PREC);
-  // per-device "attribute set" flags; a race only repeats the (idempotent) attribute call
-  static std::atomic<bool> attr_set[64];
-  int dev = 0;
-  cudaGetDevice(&dev);
-  if (!attr_set[dev & 63].load(std::memory_order_acquire)) {
-    cudaError_t e = cudaFuncSetAttribute(mlp_tc_kernel<PREC, IN_KIND>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)tc_layout(kMaxHiddenLayers, PREC).total +
-#if defined(LAKE_TRACE) && defined(LAKE_TRACE_SMEM)
-                                             (PREC == 2 ? 0 : 4 * LAKE_TRACE_CAP * 16)
-#else
-                                             0
-#endif
-                                         );
-    if (e != cudaSuccess) return e;
-    attr_set[dev & 63].store(true, std::memory_order_release);
-  }
 #if defined(LAKE_TRACE) && defined(LAKE_TRACE_SMEM)
   constexpr uint32_t kTraceBytes = PREC == 2 ? 0u : 4u * LAKE_TRACE_CAP * 16u;
 #else
   constexpr uint32_t kTraceBytes = 0;
 #endif
-  mlp_tc_kernel<PREC, IN_KIND><<<grid, kThreads, L.total + kTraceBytes, s>>>(in, ts, nh_layout, dec,
-                                                                            logits);
+  // per-device "attribute set" flags; a race only repeats the (idempotent) attribute call
+  static std::atomic<bool> attr_set[64];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (!attr_set[dev & 63].load(std::memory_order_acquire)) {
+    const uint32_t most = OTC ? tc_layout(1, PREC).total : tc_layout(kMaxHiddenLayers, PREC).total;
+    cudaError_t e = cudaFuncSetAttribute(mlp_tc_kernel<PREC, IN_KIND, OTC>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)(most + kTraceBytes));
+    if (e != cudaSuccess) return e;
+    attr_set[dev & 63].store(true, std::memory_order_release);
+  }
+  mlp_tc_kernel<PREC, IN_KIND, OTC><<<grid, kThreads, L.total + kTraceBytes, s>>>(in, ts, nh_layout,
+                                                                                 dec, logits);
   return cudaGetLastError();
+}
+
+template <int PREC, int IN_KIND>
+cudaError_t launch_o(const void *in, const TileSched &ts, int nh_layout, uint8_t *dec,
+                     float *logits, cudaStream_t s, int grid) {
+  if constexpr (out_on_tc(1, PREC))
+    if (out_on_tc(nh_layout, PREC))
+      return launch_t<PREC, IN_KIND, true>(in, ts, nh_layout, dec, logits, s, grid);
+  return launch_t<PREC, IN_KIND, false>(in, ts, nh_layout, dec, logits, s, grid);
 }
 
 template <int PREC>
 cudaError_t launch_p(const void *in, int in_kind, const TileSched &ts, int nh, uint8_t *dec,
                      float *logits, cudaStream_t s, int grid) {
-  return in_kind == LAKE_IN_RAW ? launch_t<PREC, LAKE_IN_RAW>(in, ts, nh, dec, logits, s, grid)
-                                : launch_t<PREC, LAKE_IN_DIGITS>(in, ts, nh, dec, logits, s, grid);
+  return in_kind == LAKE_IN_RAW ? launch_o<PREC, LAKE_IN_RAW>(in, ts, nh, dec, logits, s, grid)
+                                : launch_o<PREC, LAKE_IN_DIGITS>(in, ts, nh, dec, logits, s, grid);
 }
 
 }  // namespace
@@ -1194,10 +1349,13 @@ cudaError_t launch_mlp_tc(const void *in, int in_kind, int prec, const TileSched
   const int64_t clusters = ts.n_tiles < max_clusters ? ts.n_tiles : max_clusters;
   if (clusters <= 0) return cudaSuccess;
   const int grid = (int)(clusters * 2);
+  if (nh < 1 || nh > kMaxHiddenLayers) return cudaErrorInvalidValue;
+  TileSched t2 = ts;
+  t2.nh_cap = nh;
   cudaError_t e;
-  if (prec == 0) e = launch_p<0>(in, in_kind, ts, nh, decisions, logits, s, grid);
-  else if (prec == 1) e = launch_p<1>(in, in_kind, ts, nh, decisions, logits, s, grid);
-  else e = launch_p<2>(in, in_kind, ts, nh, decisions, logits, s, grid);
+  if (prec == 0) e = launch_p<0>(in, in_kind, t2, nh, decisions, logits, s, grid);
+  else if (prec == 1) e = launch_p<1>(in, in_kind, t2, nh, decisions, logits, s, grid);
+  else e = launch_p<2>(in, in_kind, t2, nh, decisions, logits, s, grid);
   count_launch();
   return e;
 }

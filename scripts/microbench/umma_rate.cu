@@ -1,6 +1,6 @@
 // Microbenchmark: cycles per tcgen05.mma.cta_group::2.kind::f16 for the operand
 // configurations the fused kernel can use (A from TMEM or SMEM, B K-major or MN-major
-// SWIZZLE_NONE, N = 128 or 256). One CTA pair, one issuing thread, 4096 MMAs back to back.
+// SWIZZLE_NONE, N = 16 .. 256). One CTA pair, one issuing thread, 4096 MMAs back to back.
 // build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 -o umma_rate umma_rate.cu
 #include <cstdio>
 #include <cstdint>
@@ -84,5 +84,10 @@ int main() {
   run<1, 0, 256, 0>("A=TMEM B=K   N=256");
   run<0, 0, 256, 0>("A=SMEM B=K   N=256");
   run<1, 1, 128, 16>("A=TMEM B=MN  N=128 sbo+16");
+  // the NN output layer (N = 16) and neighbours
+  run<1, 0, 16, 0>("A=TMEM B=K   N=16");
+  run<0, 0, 16, 0>("A=SMEM B=K   N=16");
+  run<1, 0, 32, 0>("A=TMEM B=K   N=32");
+  run<1, 0, 64, 0>("A=TMEM B=K   N=64");
   return 0;
 }
