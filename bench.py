@@ -774,6 +774,22 @@ def run_report(args):
                          inferences_per_s=round(n / (t_multi / 1e3), 1),
                          grouping_overhead=round(t_multi / t_split - 1, 4)))
         log(json.dumps(rows[-1]))
+        if arch == 0:
+            # single-model NN over 2^24 I/Os (the C4 records four times over: > 2x L2),
+            # the model LinnOS deploys, per tensor-core type
+            big = torch.from_numpy(np.ascontiguousarray(np.tile(w["raw"], (4, 1))).view(np.int32)).to(dev)
+            dbig = torch.empty(1 << 24, dtype=torch.uint8, device=dev)
+            for prec in ("f16", "bf16", "tf32"):
+                fl = lake.LAKE_IN_RAW | lake.PREC_FLAGS[prec]
+                ms = timed(lambda: lake.infer(big, fl, 1 << 24, 0, dbig, None, stream))
+                tflops = ARCH_FLOPS[0] * (1 << 24) / (ms / 1e3) / 1e12
+                gbs = (RAW_BYTES + 1) * (1 << 24) / (ms / 1e3) / 1e9
+                rows.append(dict(config="C4-single", arch="NN", path=prec, n=1 << 24, ms=round(ms, 4),
+                                 inferences_per_s=round((1 << 24) / (ms / 1e3), 1),
+                                 tflops=round(tflops, 2), frac_of_peak=round(tflops / peak_of(prec), 4),
+                                 peak=peak_label(prec), hbm_gb_s=round(gbs, 1)))
+                log(json.dumps(rows[-1]))
+            del big, dbig
         for m in w["models"]:
             lake.unload(m, 0)
         del x, ids, dec, ws, parts
