@@ -16,7 +16,11 @@ constexpr int kMaxHiddenLayers = 3;
 // Per layer l the weights are stored transposed, W^T[k][j], k < K_l, with the 256 output
 // columns permuted so that thread tc's 8 columns {tc + 32*jj} are two contiguous float4
 // groups: position p(j) = (jj/4)*128 + tc*4 + (jj%4) with tc = j%32, jj = j/32.
-constexpr int kF32TileM = 64;       // I/Os per CTA tile
+#ifndef LAKE_F32_RN
+#define LAKE_F32_RN 16  // FP32 register tile columns per thread: 16 (M 128, 1 CTA/SM) or 8 (M 64)
+#endif
+constexpr int kF32TileRN = LAKE_F32_RN;
+constexpr int kF32TileM = kF32TileRN == 16 ? 128 : 64;  // I/Os per CTA tile (mlp_fp32.cu)
 constexpr int kF32Threads = 256;
 #ifndef LAKE_F32_KC
 #define LAKE_F32_KC 16  // 2 CTAs per SM fit only with 16-row chunks (64 was best at 1 CTA/SM)

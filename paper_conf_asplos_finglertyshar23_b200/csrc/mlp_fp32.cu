@@ -39,27 +39,46 @@ constexpr int kF32ActBufs = LAKE_F32_ACT_BUFS;
 #define LAKE_F32_CTAS 2  // CTAs per SM (<= 128 registers; A/B: 1 -> 2 CTAs +3% NN+2, +36% NN)
 #endif  // 1: in place (frees SMEM for KC = 64)
 
-template <int RM>
+#ifndef LAKE_F32_PF
+#define LAKE_F32_PF 0  // 1: register double buffer of the next k-step (A/B: 6.74 vs 5.76 ms)
+#endif
+#ifndef LAKE_F32_WIDE_KC
+#define LAKE_F32_WIDE_KC 32
+#endif
+// Register tile RM rows x RN columns per thread, 256 threads: CG column groups (lanes across
+// the 256 columns) x RG row groups, M = RG * RM rows per tile.
+//   RM 2, RN 8  (M 16):  small single-model batches (latency)
+//   RM 8, RN 8  (M 64):  two CTAs per SM (round 1)
+//   RM 8, RN 16 (M 128): one CTA per SM, 128 accumulators per thread: per k-step 6 shared
+//                        loads feed 128 FFMAs (RN 8: 4 feed 64), half the SMEM wavefronts
+//                        per FMA and fewer barriers per FMA (32-row weight chunks)
+template <int RM, int RN>
 struct F32Cfg {
-  static constexpr int M = 8 * RM;                       // rows per tile
+  static constexpr int CG = 256 / RN;                    // column groups
+  static constexpr int RG = kF32Threads / CG;            // row groups
+  static constexpr int M = RG * RM;                      // rows per tile
   static constexpr int HR = RM / 2;                      // rows per thread per half-tile
+  static constexpr int NF4 = RN / 4;                     // float4 weight loads per k-step
   // activation row stride: float4-aligned with a 4-float pad for RM = 8 (conflict-free
   // float4 epilogue stores), odd for RM = 2 (conflict-free scalar stores)
-  static constexpr int S = RM == 8 ? kF32ActStride : M + 1;
-  // rows of W^T per pipeline stage (LAKE_F32_KC): 16 so that two CTAs fit per SM (A/B on
-  // B200: 1 CTA/SM with 64-row chunks 6.37 ms, 2 CTAs/SM with 16-row chunks 6.19 ms, C3 NN+2)
-  static constexpr int KC = RM == 8 ? kF32KChunk : 16;
+  static constexpr int S = RM == 8 ? M + 4 : M + 1;
+  // rows of W^T per pipeline stage: RN 8 / RM 8 uses 16 (LAKE_F32_KC) so that two CTAs fit
+  // per SM (A/B on B200: 1 CTA/SM with 64-row chunks 6.37 ms, 2 CTAs/SM with 16-row chunks
+  // 6.19 ms, C3 NN+2)
+  static constexpr int KC = RN == 16 ? LAKE_F32_WIDE_KC : (RM == 8 ? kF32KChunk : 16);
+  static constexpr int CTAS = RN == 16 ? 1 : LAKE_F32_CTAS;  // resident CTAs per SM
 };
+static_assert(F32Cfg<8, kF32TileRN>::M == kF32TileM, "multi-model FP32 tile rows");
 
-template <int RM>
+template <int RM, int RN>
 struct F32Smem {
   // transposed activations, updated in place: a layer's outputs are written only after
   // the __syncthreads that closes its last K chunk, i.e. once every input has been read
-  float act[kF32ActBufs][kHidden][F32Cfg<RM>::S];
-  float w[2][F32Cfg<RM>::KC][kHidden];   // W^T chunk staging (permuted columns)
+  float act[kF32ActBufs][kHidden][F32Cfg<RM, RN>::S];
+  float w[2][F32Cfg<RM, RN>::KC][kHidden];   // W^T chunk staging (permuted columns)
   float wout[2][kHidden];
   float bout[4];
-  int32_t rows[F32Cfg<RM>::M];           // I/O index per tile row, -1 = padding
+  int32_t rows[F32Cfg<RM, RN>::M];           // I/O index per tile row, -1 = padding
 };
 
 __device__ __forceinline__ void stage_chunk(float (*dst)[kHidden], const float *src, int rows) {
@@ -72,17 +91,18 @@ __device__ __forceinline__ void stage_chunk(float (*dst)[kHidden], const float *
   __pipeline_commit();
 }
 
-template <int IN_KIND, int RM>
-__global__ void __launch_bounds__(kF32Threads, LAKE_F32_CTAS)
+template <int IN_KIND, int RM, int RN>
+__global__ void __launch_bounds__(kF32Threads, F32Cfg<RM, RN>::CTAS)
 mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
                 uint8_t *__restrict__ decisions,
                 float *__restrict__ logits) {
-  constexpr int M = F32Cfg<RM>::M, S = F32Cfg<RM>::S, HR = F32Cfg<RM>::HR, KC = F32Cfg<RM>::KC;
+  using C = F32Cfg<RM, RN>;
+  constexpr int M = C::M, S = C::S, HR = C::HR, KC = C::KC, CG = C::CG, NF4 = C::NF4;
   extern __shared__ __align__(16) uint8_t smem_raw[];
-  F32Smem<RM> &sm = *reinterpret_cast<F32Smem<RM> *>(smem_raw);
+  F32Smem<RM, RN> &sm = *reinterpret_cast<F32Smem<RM, RN> *>(smem_raw);
   const int tid = threadIdx.x;
-  const int tr = tid >> 5;   // warp: row group
-  const int tc = tid & 31;   // lane: column group
+  const int tr = tid / CG;   // row group
+  const int tc = tid % CG;   // column group
   const int64_t n_tiles = ts.n_tiles_dev ? (int64_t)*ts.n_tiles_dev : ts.n_tiles;
 
   for (int64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
@@ -121,15 +141,16 @@ mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched t
 #pragma unroll
         for (int k = 0; k < 32; ++k) a0[k][tid] = (float)((w[k >> 2] >> ((k & 3) * 8)) & 0xFFu);
       }
-    } else if (tid < M + 2 * kHidden / 4 + 1) {
-      // output-layer weights for this tile's model
-      const int i = tid - M;
-      if (i < 2 * kHidden / 4)
-        reinterpret_cast<float4 *>(&sm.wout[0][0])[i] =
-            __ldg(reinterpret_cast<const float4 *>(mp->wout) + i);
-      else {
-        sm.bout[0] = __ldg(mp->bout);
-        sm.bout[1] = __ldg(mp->bout + 1);
+    } else {
+      // output-layer weights for this tile's model (the threads not digitising)
+      for (int i = tid - M; i <= 2 * kHidden / 4; i += kF32Threads - M) {
+        if (i < 2 * kHidden / 4)
+          reinterpret_cast<float4 *>(&sm.wout[0][0])[i] =
+              __ldg(reinterpret_cast<const float4 *>(mp->wout) + i);
+        else {
+          sm.bout[0] = __ldg(mp->bout);
+          sm.bout[1] = __ldg(mp->bout + 1);
+        }
       }
     }
     // ---- hidden layers -----------------------------------------------------------------
@@ -139,11 +160,11 @@ mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched t
       const float *wt = mp->wt[l];
       const float (*ain)[S] = sm.act[kF32ActBufs == 2 ? (l & 1) : 0];
       float (*aout)[S] = sm.act[kF32ActBufs == 2 ? ((l + 1) & 1) : 0];
-      float acc[RM][8];
+      float acc[RM][RN];
 #pragma unroll
       for (int i = 0; i < RM; ++i)
 #pragma unroll
-        for (int j = 0; j < 8; ++j) acc[i][j] = 0.0f;
+        for (int j = 0; j < RN; ++j) acc[i][j] = 0.0f;
       const int nch = (Kst + KC - 1) / KC;  // layer 0 stages its 32 rows even when KC > 32
       stage_chunk(sm.w[0], wt, Kst < KC ? Kst : KC);
       for (int c = 0; c < nch; ++c) {
@@ -157,10 +178,9 @@ mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched t
         __syncthreads();
         const float (*wc)[kHidden] = sm.w[c & 1];
         const int kmax = (K - c * KC) < KC ? (K - c * KC) : KC;
-#pragma unroll kF32Unroll
-        for (int kk = 0; kk < kmax; ++kk) {
+        // one k-step's operands: RM activations (broadcast float4 reads) and RN weights
+        auto load_ops = [&](int kk, float (&av)[RM], float (&bv)[RN]) {
           const int k = c * KC + kk;
-          float av[RM];
           if constexpr (HR == 4) {
             const float4 a0 = *reinterpret_cast<const float4 *>(&ain[k][tr * 4]);
             const float4 a1 = *reinterpret_cast<const float4 *>(&ain[k][M / 2 + tr * 4]);
@@ -173,21 +193,51 @@ mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched t
               av[HR + i] = ain[k][M / 2 + tr * HR + i];
             }
           }
-          const float4 b0 = *reinterpret_cast<const float4 *>(&wc[kk][tc * 4]);
-          const float4 b1 = *reinterpret_cast<const float4 *>(&wc[kk][128 + tc * 4]);
-          const float bv[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+#pragma unroll
+          for (int f = 0; f < NF4; ++f) {
+            const float4 b4 = *reinterpret_cast<const float4 *>(&wc[kk][f * 4 * CG + tc * 4]);
+            bv[4 * f] = b4.x; bv[4 * f + 1] = b4.y; bv[4 * f + 2] = b4.z; bv[4 * f + 3] = b4.w;
+          }
+        };
+#if LAKE_F32_PF
+        // software-pipelined: k-step kk+1's shared loads are in flight during kk's FFMAs (with
+        // two warps per scheduler at RN 16, their latency was the top stall)
+        float av[RM], bv[RN];
+        load_ops(0, av, bv);
+#pragma unroll kF32Unroll
+        for (int kk = 0; kk < kmax; ++kk) {
+          float an[RM], bn[RN];
+          if (kk + 1 < kmax) load_ops(kk + 1, an, bn);
 #pragma unroll
           for (int i = 0; i < RM; ++i)
 #pragma unroll
-            for (int j = 0; j < 8; ++j) acc[i][j] = __fmaf_rn(av[i], bv[j], acc[i][j]);
+            for (int j = 0; j < RN; ++j) acc[i][j] = __fmaf_rn(av[i], bv[j], acc[i][j]);
+#pragma unroll
+          for (int i = 0; i < RM; ++i) av[i] = an[i];
+#pragma unroll
+          for (int j = 0; j < RN; ++j) bv[j] = bn[j];
         }
+#else
+#pragma unroll kF32Unroll
+        for (int kk = 0; kk < kmax; ++kk) {
+          float av[RM], bv[RN];
+          load_ops(kk, av, bv);
+#pragma unroll
+          for (int i = 0; i < RM; ++i)
+#pragma unroll
+            for (int j = 0; j < RN; ++j) acc[i][j] = __fmaf_rn(av[i], bv[j], acc[i][j]);
+        }
+#endif
         __syncthreads();
       }
       // epilogue: z = acc + b (one rounding), ReLU, store transposed
       const float *bias = mp->b[l];
 #pragma unroll
-      for (int jj = 0; jj < 8; ++jj) {
-        const int j = tc + 32 * jj;
+      for (int jj = 0; jj < RN; ++jj) {
+        // staged position p of this accumulator column -> its neuron (the load-time column
+        // permutation: position 128 b + 4 t + q holds neuron t + 32 (q + 4 b), t < 32)
+        const int p = (jj / 4) * 4 * CG + tc * 4 + (jj % 4);
+        const int j = ((p >> 2) & 31) + 32 * ((p & 3) + 4 * (p >> 7));
         const float bj = __ldg(bias + j);
         float h[RM];
 #pragma unroll
@@ -227,21 +277,21 @@ mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched t
   }
 }
 
-template <int IN_KIND, int RM>
+template <int IN_KIND, int RM, int RN>
 cudaError_t launch_rm(const void *in, const TileSched &ts, uint8_t *decisions, float *logits,
                       cudaStream_t s, int64_t grid) {
-  const size_t smem = sizeof(F32Smem<RM>);
+  const size_t smem = sizeof(F32Smem<RM, RN>);
   static std::atomic<bool> attr_set[64];  // shared by host threads
   int dev = 0;
   cudaGetDevice(&dev);
   if (!attr_set[dev & 63].load(std::memory_order_acquire)) {
-    cudaError_t e = cudaFuncSetAttribute(mlp_fp32_kernel<IN_KIND, RM>,
+    cudaError_t e = cudaFuncSetAttribute(mlp_fp32_kernel<IN_KIND, RM, RN>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     attr_set[dev & 63].store(true, std::memory_order_release);
   }
-  mlp_fp32_kernel<IN_KIND, RM><<<(unsigned)grid, kF32Threads, smem, s>>>(in, ts, decisions,
-                                                                       logits);
+  mlp_fp32_kernel<IN_KIND, RM, RN><<<(unsigned)grid, kF32Threads, smem, s>>>(in, ts, decisions,
+                                                                           logits);
   return cudaGetLastError();
 }
 
@@ -259,16 +309,16 @@ cudaError_t launch_mlp_fp32(const void *in, int in_kind, const TileSched &ts_in,
   // small single-model batches: 16-row tiles (4x less work per tile on the critical path)
   const bool small = ts.tile_model == nullptr && ts.n <= (int64_t)16 * sms;
   if (small) ts.n_tiles = (ts.n + 15) / 16;
-  const int64_t cap = (int64_t)sms * LAKE_F32_CTAS;  // resident CTAs
+  const int64_t cap = (int64_t)sms * (small ? F32Cfg<2, 8>::CTAS : F32Cfg<8, kF32TileRN>::CTAS);
   const int64_t grid = ts.n_tiles < cap ? ts.n_tiles : cap;
   if (grid <= 0) return cudaSuccess;
   cudaError_t e;
   if (in_kind == LAKE_IN_RAW)
-    e = small ? launch_rm<LAKE_IN_RAW, 2>(in, ts, decisions, logits, s, grid)
-              : launch_rm<LAKE_IN_RAW, 8>(in, ts, decisions, logits, s, grid);
+    e = small ? launch_rm<LAKE_IN_RAW, 2, 8>(in, ts, decisions, logits, s, grid)
+              : launch_rm<LAKE_IN_RAW, 8, kF32TileRN>(in, ts, decisions, logits, s, grid);
   else
-    e = small ? launch_rm<LAKE_IN_DIGITS, 2>(in, ts, decisions, logits, s, grid)
-              : launch_rm<LAKE_IN_DIGITS, 8>(in, ts, decisions, logits, s, grid);
+    e = small ? launch_rm<LAKE_IN_DIGITS, 2, 8>(in, ts, decisions, logits, s, grid)
+              : launch_rm<LAKE_IN_DIGITS, 8, kF32TileRN>(in, ts, decisions, logits, s, grid);
   count_launch();
   return e;
 }
