@@ -24,11 +24,20 @@ for n in (1, 129, 3000):
     for f in (lake.LAKE_PREC_FP32, lake.LAKE_PREC_F16, lake.LAKE_PREC_BF16):
         lake.infer(x, lake.LAKE_IN_RAW | f, n, 3, dec, lg)
 lake.infer(d, lake.LAKE_IN_DIGITS | lake.LAKE_PREC_F16, 129, 2, dec, lg)
+# NN kernel (output layer on the tensor cores) and tf32
+for n in (1, 129, 3000):
+    for f in (lake.LAKE_PREC_F16, lake.LAKE_PREC_BF16):
+        lake.infer(x, lake.LAKE_IN_RAW | f, n, 1, dec, lg)
+    lake.infer(x, lake.LAKE_IN_RAW | lake.LAKE_PREC_TF32, n, 3, dec, lg)
+lake.infer(d, lake.LAKE_IN_DIGITS | lake.LAKE_PREC_F16, 3000, 1, dec, lg)
 ids = torch.from_numpy(np.random.default_rng(0).integers(1, 4, 3000).astype(np.int32)).to(dev)
 wsb = lake.workspace_bytes(3000)
 ws = torch.empty(wsb, dtype=torch.uint8, device=dev)
 lake.infer_multi(x, lake.LAKE_IN_RAW | lake.LAKE_PREC_F16, 3000, ids, dec, lg, ws, wsb)
 lake.infer_multi(x, lake.LAKE_IN_RAW | lake.LAKE_PREC_FP32, 3000, ids, dec, lg, ws, wsb)
+lake.infer_multi(x, lake.LAKE_IN_RAW | lake.LAKE_PREC_TF32, 3000, ids, dec, lg, ws, wsb)
+ids1 = torch.ones(3000, dtype=torch.int32, device=dev)  # NN only: one NN-layout kernel
+lake.infer_multi(x, lake.LAKE_IN_RAW | lake.LAKE_PREC_F16, 3000, ids1, dec, lg, ws, wsb)
 tr = inputs.device_trace("azure", 1000, 3, 3.0)
 a = torch.from_numpy(tr["arrival_ns"]).to(dev)
 c = torch.from_numpy(tr["complete_ns"]).to(dev)
