@@ -9,7 +9,7 @@ ARCH      := -gencode arch=compute_100a,code=sm_100a
 # --fmad=false: no implicit mul+add contraction anywhere (FP32 path is bit-exact, R15)
 NVFLAGS   := $(ARCH) -O3 -lineinfo -std=c++17 --fmad=false -Xcompiler -fPIC,-O2 \
              -Xptxas -v --expt-relaxed-constexpr
-SRCS      := $(CSRC)/api.cu $(CSRC)/digitize.cu $(CSRC)/mlp_fp32.cu $(CSRC)/mlp_tc.cu $(CSRC)/group.cu $(CSRC)/capture.cu $(CSRC)/server.cu $(CSRC)/mlp_family.cu $(CSRC)/deferred.cu
+SRCS      := $(CSRC)/api.cu $(CSRC)/digitize.cu $(CSRC)/mlp_fp32.cu $(CSRC)/mlp_tc.cu $(CSRC)/group.cu $(CSRC)/capture.cu $(CSRC)/sort.cu $(CSRC)/server.cu $(CSRC)/mlp_family.cu $(CSRC)/deferred.cu
 HDRS      := $(wildcard $(CSRC)/*.h $(CSRC)/*.cuh) include/lake_linnos.h include/lake_mlp.h
 OBJS      := $(patsubst $(CSRC)/%.cu,build/%.o,$(SRCS))
 

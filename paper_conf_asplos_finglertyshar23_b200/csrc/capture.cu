@@ -10,12 +10,10 @@
 // (every j with c_j <= a_i arrived strictly before i, so the completed count needs no
 // arrival condition).
 //
-// Device algorithm: two stable LSD radix sorts (CUB) of 63-bit keys (device << 47 | time)
-// with I/O indices as values — completions and arrivals, both ordered by (device, time,
-// index) — then one thread per I/O: a binary search of (device << 47 | a_i) in the sorted
-// completions gives the completed count and the newest four completed I/Os.
-#include <cub/device/device_radix_sort.cuh>
-
+// Device algorithm: two stable LSD radix sorts (sort.cu, hand-written) of 63-bit keys
+// (device << 47 | time) with I/O indices as values — completions and arrivals, both ordered
+// by (device, time, index) — then one thread per I/O: a binary search of (device << 47 | a_i)
+// in the sorted completions gives the completed count and the newest four completed I/Os.
 #include "lake_internal.h"
 
 namespace lake {
@@ -30,13 +28,14 @@ __device__ __forceinline__ uint64_t ckey(int32_t dev, int64_t t) {
 
 __global__ void make_keys(const int64_t *__restrict__ a, const int64_t *__restrict__ c,
                           const int32_t *__restrict__ dev, int64_t n, uint64_t *ka, uint64_t *kc,
-                          int32_t *iota) {
+                          int32_t *ic, int32_t *ia) {
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
        i += (int64_t)gridDim.x * blockDim.x) {
     const int32_t d = dev ? dev[i] : 0;
     ka[i] = ckey(d, a[i]);
     kc[i] = ckey(d, c[i]);
-    iota[i] = (int32_t)i;
+    ic[i] = (int32_t)i;
+    ia[i] = (int32_t)i;
   }
 }
 
@@ -102,10 +101,10 @@ __global__ void history(const int64_t *__restrict__ a, const int64_t *__restrict
 size_t a256(size_t x) { return (x + 255) & ~(size_t)255; }
 
 struct CapLayout {
-  size_t ka, kc, ka2, kc2, iota, ia, ic, rank, q, ub, cub, total;
+  size_t ka, kc, ka2, kc2, iota, ia, ic, rank, q, ub, sort, total;
 };
 
-CapLayout cap_layout(int64_t n, size_t cub_bytes) {
+CapLayout cap_layout(int64_t n, size_t sort_bytes) {
   CapLayout L{};
   size_t o = 0;
   L.ka = o; o += a256(n * 8);
@@ -118,31 +117,20 @@ CapLayout cap_layout(int64_t n, size_t cub_bytes) {
   L.rank = o; o += a256(n * 4);
   L.q = o; o += a256(n * 4);
   L.ub = o; o += a256(n * 8);
-  L.cub = o; o += a256(cub_bytes);
+  L.sort = o; o += a256(sort_bytes);
   L.total = o;
   return L;
-}
-
-size_t cub_temp_bytes(int64_t n) {
-  size_t bytes = 0;
-  cub::DeviceRadixSort::SortPairs(nullptr, bytes, (const uint64_t *)nullptr, (uint64_t *)nullptr,
-                                  (const int32_t *)nullptr, (int32_t *)nullptr, (int)n, 0,
-                                  kTimeBits + 16);
-  return bytes;
 }
 
 }  // namespace
 
 size_t capture_workspace_bytes(int64_t n) {
-  size_t cb = cub_temp_bytes(n);
-  if (cb == 0) cb = (size_t)n * 8 + (64u << 20);  // no device to ask: generous bound
-  return cap_layout(n, cb).total;
+  return cap_layout(n, radix_sort_workspace_bytes(n)).total;
 }
 
 cudaError_t launch_capture(const int64_t *a, const int64_t *c, const int32_t *dev, int64_t n,
                            uint32_t *raw, void *ws, size_t ws_bytes, cudaStream_t s) {
-  const size_t cb = cub_temp_bytes(n);
-  const CapLayout L = cap_layout(n, cb);
+  const CapLayout L = cap_layout(n, radix_sort_workspace_bytes(n));
   if (ws_bytes < L.total) return cudaErrorMemoryAllocation;
   uint8_t *b = static_cast<uint8_t *>(ws);
   auto U64 = [&](size_t off) { return reinterpret_cast<uint64_t *>(b + off); };
@@ -150,22 +138,26 @@ cudaError_t launch_capture(const int64_t *a, const int64_t *c, const int32_t *de
   const int threads = 256;
   const int grid = (int)((n + threads - 1) / threads < 148 * 16 ? (n + threads - 1) / threads
                                                                 : 148 * 16);
-  make_keys<<<grid, threads, 0, s>>>(a, c, dev, n, U64(L.ka), U64(L.kc), I32(L.iota));
-  size_t tb = cb;
-  cudaError_t e = cub::DeviceRadixSort::SortPairs(b + L.cub, tb, U64(L.kc), U64(L.kc2),
-                                                  I32(L.iota), I32(L.ic), (int)n, 0,
-                                                  kTimeBits + 16, s);
+  make_keys<<<grid, threads, 0, s>>>(a, c, dev, n, U64(L.ka), U64(L.kc), I32(L.ic), I32(L.ia));
+  // (device, completion, index) and (device, arrival, index) orders; 8 passes of 8 bits,
+  // so the results land back in kc / ic and ka / ia
+  bool alt_c = false, alt_a = false;
+  cudaError_t e = radix_sort_pairs(U64(L.kc), U64(L.kc2), I32(L.ic), I32(L.iota), n,
+                                   kTimeBits + 16, b + L.sort, s, &alt_c);
   if (e != cudaSuccess) return e;
-  tb = cb;
-  e = cub::DeviceRadixSort::SortPairs(b + L.cub, tb, U64(L.ka), U64(L.ka2), I32(L.iota),
-                                      I32(L.ia), (int)n, 0, kTimeBits + 16, s);
+  e = radix_sort_pairs(U64(L.ka), U64(L.ka2), I32(L.ia), I32(L.iota), n, kTimeBits + 16,
+                       b + L.sort, s, &alt_a);
   if (e != cudaSuccess) return e;
-  invert<<<grid, threads, 0, s>>>(I32(L.ia), n, I32(L.rank));
-  pending_count<<<grid, threads, 0, s>>>(a, dev, n, U64(L.kc2), I32(L.rank), I32(L.q),
+  const uint64_t *kc_sorted = alt_c ? U64(L.kc2) : U64(L.kc);
+  const int32_t *idx_c = alt_c ? I32(L.iota) : I32(L.ic);
+  const int32_t *idx_a = alt_a ? I32(L.iota) : I32(L.ia);
+  static_assert((kTimeBits + 16 + 7) / 8 % 2 == 0, "even pass count: results in place");
+  invert<<<grid, threads, 0, s>>>(idx_a, n, I32(L.rank));
+  pending_count<<<grid, threads, 0, s>>>(a, dev, n, kc_sorted, I32(L.rank), I32(L.q),
                                          reinterpret_cast<int64_t *>(b + L.ub));
-  history<<<grid, threads, 0, s>>>(a, c, n, I32(L.ic), I32(L.q),
+  history<<<grid, threads, 0, s>>>(a, c, n, idx_c, I32(L.q),
                                    reinterpret_cast<const int64_t *>(b + L.ub), raw);
-  count_launch(4 + 2 * 4);  // own kernels + CUB's onesweep passes (approximate)
+  count_launch(4);
   return cudaGetLastError();
 }
 

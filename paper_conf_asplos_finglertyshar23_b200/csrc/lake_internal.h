@@ -143,6 +143,11 @@ cudaError_t launch_mlp_fp32(const void *in, int in_kind, const TileSched &ts,
                             uint8_t *decisions, float *logits, cudaStream_t s, int device);
 cudaError_t launch_mlp_tc(const void *in, int in_kind, int prec, const TileSched &ts, int nh,
                           uint8_t *decisions, float *logits, cudaStream_t s, int device);
+// Stable LSD radix sort of (u64 key, i32 value) pairs over the low `bits` key bits (sort.cu);
+// *in_alt: the result is in the _alt buffers (odd number of 8-bit passes).
+size_t radix_sort_workspace_bytes(int64_t n);
+cudaError_t radix_sort_pairs(uint64_t *keys, uint64_t *keys_alt, int32_t *vals, int32_t *vals_alt,
+                             int64_t n, int bits, void *ws, cudaStream_t s, bool *in_alt);
 // Grouping for infer_multi (group.cu).
 size_t group_workspace_bytes(int64_t n);
 int64_t group_max_tiles(int64_t n, int tile_rows);
