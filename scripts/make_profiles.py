@@ -63,7 +63,8 @@ KEYS = ["gpu__time_duration.sum", "sm__cycles_elapsed.avg.per_second",
         "launch__shared_mem_per_block_dynamic", "sm__warps_active.avg.pct_of_peak_sustained_active",
         "smsp__issue_active.avg.pct_of_peak_sustained_active"]
 for kind, key in (("tc", "C5_f16_g1"), ("fp32", "C3_fp32_g1"), ("dig", None),
-                  ("fammllb", "FAM_mllb_g1"), ("famkml", "FAM_kml_g1"), ("scatter", None)):
+                  ("fammllb", "FAM_mllb_g1"), ("famkml", "FAM_kml_g1"), ("scatter", None),
+                  ("nn", None)):
     rep = os.path.join(src, f"full_{kind}_{tag}.ncu-rep")
     if not os.path.exists(rep):
         continue
