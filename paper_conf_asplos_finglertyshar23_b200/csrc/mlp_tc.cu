@@ -177,7 +177,9 @@ struct Layout {
 // inside any multi-model call, and the NN+1/NN+2 kernels carry none of this code.
 #ifndef LAKE_NO_OTC
 __host__ __device__ constexpr bool out_on_tc(int nh_layout, int prec) {
-  return kEpiGroups == 2 && nh_layout == 1 && prec != 2;
+  // (the in-place packing layout below assumes the default chunking: 8 chunks, 2 warps per
+  // quadrant; A/B builds with other chunkings run NN's output layer on the CUDA cores)
+  return kEpiGroups == 2 && kEpiPerQ == 2 && kChunks == 8 && nh_layout == 1 && prec != 2;
 }
 #else  // A/B switch: output layer on CUDA cores for NN too
 __host__ __device__ constexpr bool out_on_tc(int, int) { return false; }
@@ -1098,7 +1100,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           const int pos = (int)(rank * 128 + row);
           const int64_t pp = ti.begin + pos;
           const int64_t io = (ts.perm && pos < ti.count) ? (int64_t)__ldg(ts.perm + pp) : pp;
-          static_assert(kEpiCols == 16 && kChunks == 8 && kEpiPerQ == 2, "OTC packing layout");
+          static_assert(!OTC || (kEpiCols == 16 && kChunks == 8 && kEpiPerQ == 2), "OTC packing layout");
           if (ti.model != wcur) {
             // this group's W_out block, rewritten whole (the region held another model's
             // weights in between): leader CTA rows 0, 1 = W_out, zeros elsewhere. Safe here:
