@@ -343,8 +343,10 @@ __device__ __forceinline__ void epi_to_h_tmem(const uint32_t (&r)[W], const floa
   if (p[0] == 0x12345678u && p[1] == 0x9abcdef0u)
 #endif
   {
-    if constexpr (NW == 16) ptx::tmem_st_32x32b_x16(tlane_base + col0, p);
-    else ptx::tmem_st_32x32b_x8(tlane_base + col0, p);
+    if constexpr (NW == 32) ptx::tmem_st_32x32b_x32(tlane_base + col0, p);
+    else if constexpr (NW == 16) ptx::tmem_st_32x32b_x16(tlane_base + col0, p);
+    else if constexpr (NW == 8) ptx::tmem_st_32x32b_x8(tlane_base + col0, p);
+    else ptx::tmem_st_32x32b_x4(tlane_base + col0, p);
   }
 }
 
