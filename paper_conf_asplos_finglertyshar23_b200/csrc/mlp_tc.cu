@@ -448,6 +448,39 @@ __device__ __forceinline__ void row_from_canonical(const uint32_t (&dg)[32], XRo
 // Last hidden layer: ReLU(acc + b) in fp32, accumulated straight into the two logits
 // (two partial sums per logit to halve the dependent-FMA chain). fp16/bf16: b is already
 // in acc (bias MMA).
+#ifdef LAKE_LOGITS_FFMA2
+// A/B: paired form (fma.rn.f32x2): p[0]/p[2] and p[1]/p[3] are the two lanes of one 64-bit
+// accumulator each, so every lane does exactly the scalar form's FMAs (same bits) in half the
+// FMA issue slots. Measured slower at C5 (3.287 vs 3.264 ms): the packing moves cost more.
+template <int PREC, int W>
+__device__ __forceinline__ void epi_to_logits(const uint32_t (&r)[W], const float *bl,
+                                              const float *wo, uint32_t col0, float (&p)[4]) {
+  uint64_t a0 = ptx::pack_f32x2(p[0], p[2]), a1 = ptx::pack_f32x2(p[1], p[3]);
+#pragma unroll
+  for (int c4 = 0; c4 < W / 4; ++c4) {
+    float bb[4] = {0.0f, 0.0f, 0.0f, 0.0f};
+    if constexpr (PREC == 2) {
+      const float4 b4 = *reinterpret_cast<const float4 *>(bl + col0 + c4 * 4);
+      bb[0] = b4.x; bb[1] = b4.y; bb[2] = b4.z; bb[3] = b4.w;
+    }
+    const ulonglong2 w0 = *reinterpret_cast<const ulonglong2 *>(wo + col0 + c4 * 4);
+    const ulonglong2 w1 = *reinterpret_cast<const ulonglong2 *>(wo + kHidden + col0 + c4 * 4);
+    float h[4];
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      const float v = PREC == 2 ? __uint_as_float(r[c4 * 4 + e]) + bb[e] : __uint_as_float(r[c4 * 4 + e]);
+      h[e] = v > 0.0f ? v : 0.0f;
+    }
+    const uint64_t h01 = ptx::pack_f32x2(h[0], h[1]), h23 = ptx::pack_f32x2(h[2], h[3]);
+    ptx::fma_f32x2(a0, h01, w0.x);
+    ptx::fma_f32x2(a1, h01, w1.x);
+    ptx::fma_f32x2(a0, h23, w0.y);
+    ptx::fma_f32x2(a1, h23, w1.y);
+  }
+  ptx::unpack_f32x2(a0, p[0], p[2]);
+  ptx::unpack_f32x2(a1, p[1], p[3]);
+}
+#else
 template <int PREC, int W>
 __device__ __forceinline__ void epi_to_logits(const uint32_t (&r)[W], const float *bl,
                                               const float *wo, uint32_t col0, float (&p)[4]) {
@@ -475,6 +508,7 @@ __device__ __forceinline__ void epi_to_logits(const uint32_t (&r)[W], const floa
     }
   }
 }
+#endif
 
 template <int PREC, int IN_KIND, bool OTC>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
