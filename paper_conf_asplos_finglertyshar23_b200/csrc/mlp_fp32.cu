@@ -54,21 +54,26 @@ constexpr int kF32ActBufs = LAKE_F32_ACT_BUFS;
 //                        per FMA and fewer barriers per FMA (32-row weight chunks)
 template <int RM, int RN>
 struct F32Cfg {
+  static constexpr int T = RM == 4 ? 512 : kF32Threads;  // threads (RM 4: 16 warps per CTA)
   static constexpr int CG = 256 / RN;                    // column groups
-  static constexpr int RG = kF32Threads / CG;            // row groups
+  static constexpr int RG = T / CG;                      // row groups
   static constexpr int M = RG * RM;                      // rows per tile
   static constexpr int HR = RM / 2;                      // rows per thread per half-tile
   static constexpr int NF4 = RN / 4;                     // float4 weight loads per k-step
   // activation row stride: float4-aligned with a 4-float pad for RM = 8 (conflict-free
   // float4 epilogue stores), odd for RM = 2 (conflict-free scalar stores)
-  static constexpr int S = RM == 8 ? M + 4 : M + 1;
+  static constexpr int S = RM >= 4 ? M + 4 : M + 1;
   // rows of W^T per pipeline stage: RN 8 / RM 8 uses 16 (LAKE_F32_KC) so that two CTAs fit
   // per SM (A/B on B200: 1 CTA/SM with 64-row chunks 6.37 ms, 2 CTAs/SM with 16-row chunks
   // 6.19 ms, C3 NN+2)
   static constexpr int KC = RN == 16 ? LAKE_F32_WIDE_KC : (RM == 8 ? kF32KChunk : 16);
   static constexpr int CTAS = RN == 16 ? 1 : LAKE_F32_CTAS;  // resident CTAs per SM
 };
-static_assert(F32Cfg<8, kF32TileRN>::M == kF32TileM, "multi-model FP32 tile rows");
+#ifndef LAKE_F32_RM
+#define LAKE_F32_RM 8  // rows per thread of the full-size tile: 8 (256 threads) or 4 (512 threads)
+#endif
+constexpr int kF32TileRM = LAKE_F32_RM;
+static_assert(F32Cfg<kF32TileRM, kF32TileRN>::M == kF32TileM, "multi-model FP32 tile rows");
 
 template <int RM, int RN>
 struct F32Smem {
@@ -81,10 +86,11 @@ struct F32Smem {
   int32_t rows[F32Cfg<RM, RN>::M];           // I/O index per tile row, -1 = padding
 };
 
+template <int T>
 __device__ __forceinline__ void stage_chunk(float (*dst)[kHidden], const float *src, int rows) {
   // rows x 256 floats, contiguous in global; 16-byte cp.async per thread-iteration.
   const int n16 = rows * kHidden / 4;
-  for (int i = threadIdx.x; i < n16; i += kF32Threads) {
+  for (int i = threadIdx.x; i < n16; i += T) {
     __pipeline_memcpy_async(reinterpret_cast<float4 *>(&dst[0][0]) + i,
                             reinterpret_cast<const float4 *>(src) + i, 16);
   }
@@ -92,12 +98,12 @@ __device__ __forceinline__ void stage_chunk(float (*dst)[kHidden], const float *
 }
 
 template <int IN_KIND, int RM, int RN>
-__global__ void __launch_bounds__(kF32Threads, F32Cfg<RM, RN>::CTAS)
+__global__ void __launch_bounds__(F32Cfg<RM, RN>::T, F32Cfg<RM, RN>::CTAS)
 mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
                 uint8_t *__restrict__ decisions,
                 float *__restrict__ logits) {
   using C = F32Cfg<RM, RN>;
-  constexpr int M = C::M, S = C::S, HR = C::HR, KC = C::KC, CG = C::CG, NF4 = C::NF4;
+  constexpr int M = C::M, S = C::S, HR = C::HR, KC = C::KC, CG = C::CG, NF4 = C::NF4, T = C::T;
   extern __shared__ __align__(16) uint8_t smem_raw[];
   F32Smem<RM, RN> &sm = *reinterpret_cast<F32Smem<RM, RN> *>(smem_raw);
   const int tid = threadIdx.x;
@@ -143,7 +149,7 @@ mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched t
       }
     } else {
       // output-layer weights for this tile's model (the threads not digitising)
-      for (int i = tid - M; i <= 2 * kHidden / 4; i += kF32Threads - M) {
+      for (int i = tid - M; i <= 2 * kHidden / 4; i += T - M) {
         if (i < 2 * kHidden / 4)
           reinterpret_cast<float4 *>(&sm.wout[0][0])[i] =
               __ldg(reinterpret_cast<const float4 *>(mp->wout) + i);
@@ -166,11 +172,11 @@ mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched t
 #pragma unroll
         for (int j = 0; j < RN; ++j) acc[i][j] = 0.0f;
       const int nch = (Kst + KC - 1) / KC;  // layer 0 stages its 32 rows even when KC > 32
-      stage_chunk(sm.w[0], wt, Kst < KC ? Kst : KC);
+      stage_chunk<T>(sm.w[0], wt, Kst < KC ? Kst : KC);
       for (int c = 0; c < nch; ++c) {
         if (c + 1 < nch) {
           const int rows = (Kst - (c + 1) * KC) < KC ? (Kst - (c + 1) * KC) : KC;
-          stage_chunk(sm.w[(c + 1) & 1], wt + (int64_t)(c + 1) * KC * kHidden, rows);
+          stage_chunk<T>(sm.w[(c + 1) & 1], wt + (int64_t)(c + 1) * KC * kHidden, rows);
           __pipeline_wait_prior(1);
         } else {
           __pipeline_wait_prior(0);
@@ -186,6 +192,10 @@ mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched t
             const float4 a1 = *reinterpret_cast<const float4 *>(&ain[k][M / 2 + tr * 4]);
             av[0] = a0.x; av[1] = a0.y; av[2] = a0.z; av[3] = a0.w;
             av[4] = a1.x; av[5] = a1.y; av[6] = a1.z; av[7] = a1.w;
+          } else if constexpr (HR == 2 && RM == 4) {
+            const float2 a0 = *reinterpret_cast<const float2 *>(&ain[k][tr * 2]);
+            const float2 a1 = *reinterpret_cast<const float2 *>(&ain[k][M / 2 + tr * 2]);
+            av[0] = a0.x; av[1] = a0.y; av[2] = a1.x; av[3] = a1.y;
           } else {
 #pragma unroll
             for (int i = 0; i < HR; ++i) {
@@ -249,6 +259,9 @@ mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched t
           *reinterpret_cast<float4 *>(&aout[j][tr * 4]) = make_float4(h[0], h[1], h[2], h[3]);
           *reinterpret_cast<float4 *>(&aout[j][M / 2 + tr * 4]) =
               make_float4(h[4], h[5], h[6], h[7]);
+        } else if constexpr (HR == 2 && RM == 4) {
+          *reinterpret_cast<float2 *>(&aout[j][tr * 2]) = make_float2(h[0], h[1]);
+          *reinterpret_cast<float2 *>(&aout[j][M / 2 + tr * 2]) = make_float2(h[2], h[3]);
         } else {
 #pragma unroll
           for (int i = 0; i < HR; ++i) {
@@ -290,8 +303,8 @@ cudaError_t launch_rm(const void *in, const TileSched &ts, uint8_t *decisions, f
     if (e != cudaSuccess) return e;
     attr_set[dev & 63].store(true, std::memory_order_release);
   }
-  mlp_fp32_kernel<IN_KIND, RM, RN><<<(unsigned)grid, kF32Threads, smem, s>>>(in, ts, decisions,
-                                                                           logits);
+  mlp_fp32_kernel<IN_KIND, RM, RN><<<(unsigned)grid, F32Cfg<RM, RN>::T, smem, s>>>(in, ts, decisions,
+                                                                                 logits);
   return cudaGetLastError();
 }
 
@@ -309,16 +322,16 @@ cudaError_t launch_mlp_fp32(const void *in, int in_kind, const TileSched &ts_in,
   // small single-model batches: 16-row tiles (4x less work per tile on the critical path)
   const bool small = ts.tile_model == nullptr && ts.n <= (int64_t)16 * sms;
   if (small) ts.n_tiles = (ts.n + 15) / 16;
-  const int64_t cap = (int64_t)sms * (small ? F32Cfg<2, 8>::CTAS : F32Cfg<8, kF32TileRN>::CTAS);
+  const int64_t cap = (int64_t)sms * (small ? F32Cfg<2, 8>::CTAS : F32Cfg<kF32TileRM, kF32TileRN>::CTAS);
   const int64_t grid = ts.n_tiles < cap ? ts.n_tiles : cap;
   if (grid <= 0) return cudaSuccess;
   cudaError_t e;
   if (in_kind == LAKE_IN_RAW)
     e = small ? launch_rm<LAKE_IN_RAW, 2, 8>(in, ts, decisions, logits, s, grid)
-              : launch_rm<LAKE_IN_RAW, 8, kF32TileRN>(in, ts, decisions, logits, s, grid);
+              : launch_rm<LAKE_IN_RAW, kF32TileRM, kF32TileRN>(in, ts, decisions, logits, s, grid);
   else
     e = small ? launch_rm<LAKE_IN_DIGITS, 2, 8>(in, ts, decisions, logits, s, grid)
-              : launch_rm<LAKE_IN_DIGITS, 8, kF32TileRN>(in, ts, decisions, logits, s, grid);
+              : launch_rm<LAKE_IN_DIGITS, kF32TileRM, kF32TileRN>(in, ts, decisions, logits, s, grid);
   count_launch();
   return e;
 }
