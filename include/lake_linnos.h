@@ -102,7 +102,11 @@ enum lake_flags {
     LAKE_IN_RAW     = 0x01, /* in = const lake_io_raw_t[n]; digitised inside the kernel  */
     LAKE_PREC_FP32  = 0x00, /* CUDA-core FP32, strict operation order: bit-exact with the
                                oracle (DESIGN.md §3 reading R15)                           */
-    LAKE_PREC_F16   = 0x10, /* tcgen05 tensor cores, fp16 operands, fp32 accumulation     */
+    LAKE_PREC_F16   = 0x10, /* tcgen05 tensor cores, fp16 operands, fp32 accumulation;
+                               NN (one hidden layer) also runs its 2-wide output layer on
+                               the tensor cores (fp16 H and W_out), NN+1 / NN+2 in fp32 on
+                               CUDA cores; an NN I/O gets the same bits in single- and
+                               multi-model calls                         */
     LAKE_PREC_BF16  = 0x20, /* tcgen05 tensor cores, bf16 operands, fp32 accumulation;
                                8 mantissa bits: reported, below the north_star agreement
                                bar on the synthetic models                  */
