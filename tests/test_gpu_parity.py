@@ -499,6 +499,22 @@ def test_capture_equals_oracle(quantum):
     assert np.array_equal(_gpu_capture(a, c, d), oracle.capture(a, c, d))
 
 
+def test_capture_shuffled_wide_devices_and_ties():
+    # the hand-written radix sort (csrc/sort.cu) over every digit: input in random order,
+    # device ids spanning the 16-bit range (the key's top digits), arrival/completion times
+    # spread over the full 47 bits and quantised to 1 ms (many equal keys: stability)
+    rng = np.random.default_rng(123)
+    n = 50_000
+    devs = np.array([0, 1, 255, 256, 4097, 65535], np.int32)
+    d = devs[rng.integers(0, devs.size, n)]
+    base = rng.integers(0, 1 << 44, devs.size)  # per-device epoch: high time digits in play
+    a = base[np.searchsorted(devs, d)] + rng.integers(0, 200, n) * 1_000_000
+    c = a + 1 + rng.integers(0, 5, n) * 1_000_000
+    assert int(c.max()) < (1 << 47)
+    got = _gpu_capture(a.astype(np.int64), c.astype(np.int64), d)
+    assert np.array_equal(got, oracle.capture(a.astype(np.int64), c.astype(np.int64), d))
+
+
 def test_capture_full_size_sampled():
     a, c, d = _interleaved_trace(1 << 20, 8, seed=80)
     got = _gpu_capture(a, c, d)
