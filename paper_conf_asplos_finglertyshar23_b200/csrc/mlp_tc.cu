@@ -199,6 +199,28 @@ constexpr uint32_t kWoutBytes = 8u * kHidden * 2;    // one group's W_out block 
 constexpr uint32_t kLboR8 = 8 * 16;                  // K-direction core stride, 8-row operand
 constexpr uint32_t kOutDCol = kHidden - 16;          // output accumulator: columns 240..255
 constexpr uint32_t kOutLastA = 13 * 16 + 8;          // last K-step's packed H: K-step 13's gap
+// Split of the NN output layer's K = 256 between the tensor cores and the CUDA cores: K-steps
+// [0, kOtcKs) (features 0 .. 16 kOtcKs - 1, chunks j < kOtcKs / 2) are packed and multiplied
+// by N = 16 MMAs; the rest are ReLU'd and dotted with W_out in fp32 by the draining group
+// while it would otherwise wait for those MMAs. A narrow MMA costs >= 62 cycles whatever its
+// N (scripts/microbench/umma_dep.cu: per instruction, not an accumulator dependency), so with
+// all 16 K-steps on the tensor cores the output layer (~1.3k tensor cycles per tile under
+// load) bound the NN kernel.
+#ifndef LAKE_OTC_KSTEPS
+#define LAKE_OTC_KSTEPS 16
+#endif
+constexpr uint32_t kOtcKs = LAKE_OTC_KSTEPS;
+static_assert(kOtcKs >= 4 && kOtcKs <= 16 && kOtcKs % 2 == 0, "whole chunks on the tensor cores");
+// With a CUDA-core share (kOtcKs < 16) the group packs the tensor chunks, arrives on HDONE
+// and then does the CUDA chunks while the output MMAs run; those chunks' columns are still
+// fp32 H, so the output accumulator moves to columns 24..39, freed by packing chunks 0 and 1
+// "shifted": the first warp of the quadrant packs its 16 columns into its own second half
+// (32j + 8), the second into its own first half (32j + 16), leaving 32j+24 .. 32j+40 free.
+constexpr uint32_t kOtcDCol = kOtcKs == 16 ? kOutDCol : 24u;
+__host__ __device__ constexpr uint32_t otc_a_col(uint32_t ks) {
+  return kOtcKs == 16 ? (ks + 1 == kHidden / 16 ? kOutLastA : ks * 16)
+                      : (ks < 4 && (ks & 1) == 0 ? ks * 16 + 8 : ks * 16);
+}
 __host__ __device__ constexpr uint32_t otc_wout(int prec) { return tc_w0_half_bytes(prec); }
 __host__ __device__ constexpr uint32_t otc_end(int prec) { return otc_wout(prec) + 2 * kWoutBytes; }
 
@@ -285,6 +307,27 @@ constexpr uint32_t kWarpDig = 1;
 constexpr uint32_t kWarpLoad = 3;
 constexpr uint32_t kWarpEpi = 4;
 #endif
+// A/B switch for the NN kernels with the output layer on the tensor cores (traces show their
+// MMA issuer waiting on XFULL): kOtcDigWarps digitiser warps (1 row per thread with 4), the
+// extra ones above the MMA warp (warps kThreads / 32 ..), or all of them there with
+// LAKE_OTC_DIG_TOP (warps 0-1 then idle), where the scheduler's highest-id-first arbitration
+// serves them before the epilogue. Measured slower (C4 NN pre-split 0.2418 ms with 2 warps
+// at 0-1; 4 at the top 0.2556, 2 at the top 0.2513, 4 split 0.2564): the layer-0 -> epilogue
+// -> output-MMA chain and the narrow MMAs bound these kernels, not digitiser issue slots.
+#ifndef LAKE_OTC_DIG_WARPS
+#define LAKE_OTC_DIG_WARPS 2
+#endif
+#ifndef LAKE_OTC_DIG_TOP
+#define LAKE_OTC_DIG_TOP 0
+#endif
+constexpr uint32_t kOtcDigWarps = LAKE_OTC_DIG_WARPS;
+static_assert(kOtcDigWarps == 2 || kOtcDigWarps == 4, "128 rows over 64 or 128 digitiser threads");
+constexpr bool kOtcDigTop = LAKE_OTC_DIG_TOP != 0;
+template <bool OTC> constexpr uint32_t dig_warps() { return OTC ? kOtcDigWarps : 2u; }
+template <bool OTC> constexpr uint32_t extra_warps() {
+  return OTC ? (kOtcDigTop ? kOtcDigWarps : kOtcDigWarps - 2u) : 0u;
+}
+template <bool OTC> constexpr int threads_of() { return kThreads + 32 * (int)extra_warps<OTC>(); }
 
 __device__ __forceinline__ uint32_t img_wh(int l, int prec) { return tc_wh_off(l, prec); }
 
@@ -511,7 +554,7 @@ __device__ __forceinline__ void epi_to_logits(const uint32_t (&r)[W], const floa
 #endif
 
 template <int PREC, int IN_KIND, bool OTC>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(threads_of<OTC>(), 1)
 mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts, int nh_layout,
               uint8_t *__restrict__ decisions, float *__restrict__ logits) {
   extern __shared__ __align__(1024) uint8_t smem[];
@@ -537,6 +580,11 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
                       : (warp == kWarpEpi && rank == 0) ? 1
                       : (warp == kWarpEpi && rank == 1) ? 2
                       : (warp == kWarpEpi + 4 && rank == 0) ? 3 : -1;
+#elif defined(LAKE_TRACE_OTC)  // streams: MMA, the two epilogue groups' poller warps (rank 0), digitiser
+  int tr_stream = !(tr_buf && cid == 0 && rank == 0) || lane != 0 ? -1
+                      : warp == kWarpMma ? 0 : warp == kWarpEpi + 1 ? 1
+                      : warp == kWarpEpi + kGroupWarps + 1 ? 2
+                      : threadIdx.x == ((OTC && kOtcDigTop) ? (uint32_t)kThreads : 0u) ? 3 : -1;
 #elif defined(LAKE_TRACE_DIG)  // streams: MMA, digitiser thread 0 of rank 0 / rank 1, epi warp 3
   int tr_stream = !(tr_buf && cid == 0) ? -1
                       : (warp == kWarpMma && lane == 0 && rank == 0) ? 0
@@ -845,7 +893,9 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         __syncwarp();
       }
     }
-  } else if (warp >= kWarpDig && warp < kWarpDig + 2) {
+  } else if (OTC ? (kOtcDigTop ? warp >= (uint32_t)kThreads / 32
+                                : (warp >= kWarpDig && warp < kWarpDig + 2) || warp >= (uint32_t)kThreads / 32)
+                 : (warp >= kWarpDig && warp < kWarpDig + 2)) {
     // ================= digitisers: input rows -> X (operand-type digits) ===============
     // Each CTA's 128 rows of a tile are contiguous in one of three staged formats, brought
     // into SMEM by a bulk copy (cp.async.bulk, TMA engine) two tiles ahead and converted from
@@ -856,7 +906,11 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
     //   digits  single-model calls, LAKE_IN_DIGITS, 16-B aligned input: 32-B rows
     // Anything else (misaligned input, or rows too large for this precision's staging
     // buffers) gathers each row with global loads (the fallback below).
-    const uint32_t d = threadIdx.x - kWarpDig * 32;  // 0..63
+    constexpr uint32_t ND = 32 * dig_warps<OTC>();  // digitiser threads
+    constexpr uint32_t RPT = 128 / ND;                // rows per thread: d, d + ND
+    const uint32_t d = (OTC && kOtcDigTop) ? threadIdx.x - (uint32_t)kThreads
+                       : warp < (uint32_t)kThreads / 32 ? threadIdx.x - kWarpDig * 32
+                                                        : 64u + threadIdx.x - (uint32_t)kThreads;
     const uint32_t xfull_leader0 = ptx::mapa(bar(B_XFULL), 0);
     const uint32_t row_bytes = ts.pdig ? 16u : (IN_KIND == LAKE_IN_RAW ? 36u : 32u);
 #ifdef LAKE_ABL_NOSTAGE  // A/B switch: always the gather path
@@ -895,12 +949,12 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       const TileInfo ti = tile_info<PREC>(ts, t);
       const uint32_t xb = (uint32_t)(it & 1);
       const uint32_t rows = rows_of(ti);
-      XRow<PREC> xr[2];  // rows d and d + 64 in the slot order
+      XRow<PREC> xr[RPT];  // rows d (and d + 64) in the slot order
       if (staged) {
         const uint32_t sb = (uint32_t)(it & 1);
 #ifndef LAKE_DIG_POLL_ALL
         if (d < 32) ptx::mbar_wait(bar(B_SFULL + sb), (uint32_t)((it >> 1) & 1));
-        ptx::named_bar_sync(1, 64);
+        ptx::named_bar_sync(1, ND);
 #else
         ptx::mbar_wait(bar(B_SFULL + sb), (uint32_t)((it >> 1) & 1));
 #endif
@@ -908,8 +962,8 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         const uint32_t bulk = (rows * row_bytes) & ~15u;
         const uint8_t *st = smem + L.stage + sb * kStageBytes(PREC);
 #pragma unroll
-        for (int half = 0; half < 2; ++half) {
-          const uint32_t r = d + 64 * half;
+        for (int half = 0; half < (int)RPT; ++half) {
+          const uint32_t r = d + ND * half;
           const bool valid = r < rows;
 #ifdef LAKE_ABL_NODIG  // timing-only ablation: no digitiser conversion (staged inputs)
 #pragma unroll
@@ -950,7 +1004,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         }
 #ifndef LAKE_DIG_POLL_ALL  // one polling warp (see the epilogue's accumulator-full wait)
         if (d < 32) ptx::mbar_wait(bar(B_XEMPTY + xb), (uint32_t)(((it >> 1) & 1) ^ 1));
-        ptx::named_bar_sync(1, 64);
+        ptx::named_bar_sync(1, ND);
 #else
         ptx::mbar_wait(bar(B_XEMPTY + xb), (uint32_t)(((it >> 1) & 1) ^ 1));
 #endif
@@ -958,13 +1012,13 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       } else {
         // gather fallback: both rows' loads are issued before any shared store (the
         // st.shared asm carries a memory clobber, so later loads could not be hoisted)
-        uint32_t rec[2][9];
+        uint32_t rec[RPT][9];
         // NN tiles (one tensor-core layer) are digitiser-bound: gather first, then wait.
         const bool early = ti.nh == 1;
         if (!early) ptx::mbar_wait(bar(B_XEMPTY + xb), (uint32_t)(((it >> 1) & 1) ^ 1));
 #pragma unroll
-        for (int half = 0; half < 2; ++half) {
-          const uint32_t r = d + 64 * half;
+        for (int half = 0; half < (int)RPT; ++half) {
+          const uint32_t r = d + ND * half;
           const bool valid = r < rows;
           const int64_t p = ti.begin + rank * 128 + (valid ? r : 0);
           const int64_t io = ts.perm ? (int64_t)ts.perm[p] : p;
@@ -988,7 +1042,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         if (early) ptx::mbar_wait(bar(B_XEMPTY + xb), (uint32_t)(((it >> 1) & 1) ^ 1));
         LAKE_TEV(T_XEMPTY, it, 0, 0);
 #pragma unroll
-        for (int half = 0; half < 2; ++half) {
+        for (int half = 0; half < (int)RPT; ++half) {
           if (IN_KIND == LAKE_IN_RAW) {
             row_from_raw<PREC>(rec[half], t100, xr[half]);
           } else {
@@ -1003,8 +1057,8 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       // gathered invalid rows read 0s above)
       const uint32_t xs = sbase + L.x + xb * kXB;
 #pragma unroll
-      for (int half = 0; half < 2; ++half) {
-        const uint32_t r = d + 64 * half;
+      for (int half = 0; half < (int)RPT; ++half) {
+        const uint32_t r = d + ND * half;
         constexpr int NKG = PREC == 2 ? 8 : 4;  // 16-B core-matrix groups per row
 #pragma unroll
         for (int kg = 0; kg < NKG; ++kg)
@@ -1012,7 +1066,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
                             xr[half].w[kg * 4 + 1], xr[half].w[kg * 4 + 2], xr[half].w[kg * 4 + 3]);
       }
       ptx::fence_proxy_async_smem();
-      ptx::named_bar_sync(1, 64);  // X written; staging buffer it&1 fully read
+      ptx::named_bar_sync(1, ND);  // X written; staging buffer it&1 fully read
       if (d == 0) {
         ptx::mbar_arrive_cluster(xfull_leader0 + xb * 8);
         if (staged && t + 2 < t_end) issue(t + 2, (uint32_t)(it & 1));
@@ -1204,6 +1258,28 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
             ptx::fence_proxy_async_smem();  // read by the output MMA (after the HDONE arrive)
             wcur = ti.model;
           }
+          float p[4] = {0.0f, 0.0f, 0.0f, 0.0f};  // CUDA-core share of the output layer
+          constexpr uint32_t JT = kOtcKs / 2;     // chunks (of this warp) on the tensor cores
+          // this group's leader-CTA poller: wait until both CTAs' groups packed H, then issue
+          // the output layer (A = the packed H in place, D = kOtcDCol)
+          auto issue_out = [&]() {
+            ptx::mbar_wait(bar(B_HDONE + b), (hd_phase >> b) & 1);
+            LAKE_TEV(T_OHDONE, it, b, 0);
+            ptx::tc_fence_after();
+            const bool issuer = lane == 0;
+            const uint32_t tm = __shfl_sync(0xffffffffu, tmem, 0);
+            const uint32_t idesc_out = ptx::umma_idesc_f16(PREC, 256, 16);
+            const uint64_t wd = ptx::umma_desc(sbase + L.wout + gy * kWoutBytes, kLboR8, 1024);
+            const uint32_t acc = tm + b * 256;
+#pragma unroll
+            for (uint32_t ks = 0; ks < kOtcKs; ++ks)
+              if (issuer)
+                ptx::mma_cg2_ts<PREC>(acc + kOtcDCol, acc + otc_a_col(ks),
+                                      wd + ks * ((2 * kLboR8) >> 4), idesc_out, ks);
+            if (issuer) ptx::mma_commit_cg2(bar(B_DOUT + b), 0x3);
+            __syncwarp();
+            LAKE_TEV(T_OCOMMIT, it, b, 0);
+          };
 #pragma unroll kEpiUnroll
           for (uint32_t j = 0; j < kWarpChunks; ++j) {
             const uint32_t col0 = col_of(j);
@@ -1211,36 +1287,37 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
               if (j & 1) ptx::tmem_ld_cols<W>(tbase + col_of(j + 1), ra);
               else ptx::tmem_ld_cols<W>(tbase + col_of(j + 1), rb);
             }
-            // the last K-step (chunk 7, second half) lands in K-step 13's free half, which
-            // this warp read in chunk 6; columns 240..255 stay free for the output MMA
-            const uint32_t dst = (j == kWarpChunks - 1 && hh == 1) ? kOutLastA : col0;
-            if (j & 1) epi_to_h_tmem<PREC, W>(rb, hbias, dst, tbase);
-            else epi_to_h_tmem<PREC, W>(ra, hbias, dst, tbase);
+            if (j < JT) {
+              // K-steps 2j, 2j+1 on the tensor cores, packed where otc_a_col says. With all
+              // 16 there: the last K-step (chunk 7, second half) lands in K-step 13's free
+              // half, which this warp read in chunk 6; columns 240..255 stay free for the
+              // output MMA. With fewer: chunks 0 and 1 packed shifted (see kOtcDCol)
+              const uint32_t dst = kOtcKs == 16 ? ((j == kWarpChunks - 1 && hh == 1) ? kOutLastA : col0)
+                                                : ((j < 2 && hh == 0) ? col0 + 8 : col0);
+              if (j & 1) epi_to_h_tmem<PREC, W>(rb, hbias, dst, tbase);
+              else epi_to_h_tmem<PREC, W>(ra, hbias, dst, tbase);
+            } else {
+              // on the CUDA cores (fp32; the staged last-layer bias is zero: b0 came from the
+              // MMA), after this warp's HDONE arrive: the output MMAs neither read nor write
+              // these columns
+              if (j & 1) epi_to_logits<PREC, W>(rb, prm, wo, col0, p);
+              else epi_to_logits<PREC, W>(ra, prm, wo, col0, p);
+            }
+            if (j + 1 == JT) {
+              ptx::tmem_st_wait();
+              ptx::tc_fence_before();
+              __syncwarp();
+              if (lane == 0) ptx::mbar_arrive_cluster(hdone_leader0 + b * 8);
+              LAKE_TEV(T_EHDONE, it, b, warp);
+              if (rank == 0 && lw == 1) issue_out();
+            }
             if (j + 1 < kWarpChunks) ptx::tmem_ld_wait();
           }
-          ptx::tmem_st_wait();
-          ptx::tc_fence_before();
-          __syncwarp();
-          if (lane == 0) ptx::mbar_arrive_cluster(hdone_leader0 + b * 8);
-          LAKE_TEV(T_EHDONE, it, b, warp);
-          if (rank == 0 && lw == 1) {
-            ptx::mbar_wait(bar(B_HDONE + b), (hd_phase >> b) & 1);
-            ptx::tc_fence_after();
-            const bool issuer = lane == 0;
-            const uint32_t tm = __shfl_sync(0xffffffffu, tmem, 0);
-            const uint32_t idesc_out = ptx::umma_idesc_f16(PREC, 256, 16);
-            // this group's W_out block; A = the packed H in place (K-step 15 moved: kOutLastA)
-            const uint64_t wd = ptx::umma_desc(sbase + L.wout + gy * kWoutBytes, kLboR8, 1024);
-            const uint32_t acc = tm + b * 256;
-#pragma unroll
-            for (uint32_t ks = 0; ks < kHidden / 16; ++ks)
-              if (issuer)
-                ptx::mma_cg2_ts<PREC>(acc + kOutDCol,
-                                      acc + (ks + 1 == kHidden / 16 ? kOutLastA : tmem_a_col<PREC>(ks)),
-                                      wd + ks * ((2 * kLboR8) >> 4), idesc_out, ks);
-            if (issuer) ptx::mma_commit_cg2(bar(B_DOUT + b), 0x3);
-            __syncwarp();
-            LAKE_TEV(T_OCOMMIT, it, b, 0);
+          float p0 = p[0] + p[2], p1 = p[1] + p[3];
+          if (kOtcKs < 16 && hh > 0) {  // partials of the quadrant's second warp (read below,
+            float *rd = red + row * 2;     // after the group barrier that follows DOUT)
+            rd[0] = p0;
+            rd[1] = p1;
           }
           hd_phase ^= (1u << b);
           if (lw == 1) ptx::mbar_wait(bar(B_DOUT + b), (do_phase >> b) & 1);
@@ -1250,7 +1327,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           ptx::tc_fence_after();
           uint32_t o[2] = {0u, 0u};
           if (hh == 0) {
-            ptx::tmem_ld_32x32b_x2(tbase + kOutDCol, o);
+            ptx::tmem_ld_32x32b_x2(tbase + kOtcDCol, o);
             ptx::tmem_ld_wait();
           }
           ptx::tc_fence_before();
@@ -1258,8 +1335,13 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           release_acc(b);
           LAKE_TEV(T_ETEMPTY, it, b, warp);
           if (hh == 0 && pos < ti.count) {
-            const float l0 = __uint_as_float(o[0]) + wo[2 * kHidden + 0];
-            const float l1 = __uint_as_float(o[1]) + wo[2 * kHidden + 1];
+            if (kOtcKs < 16) {
+              p0 += red[row * 2 + 0];  // the quadrant's second warp (written before the barrier)
+              p1 += red[row * 2 + 1];
+            }
+            // tensor-core share + this warp's + the second warp's CUDA-core shares + b_out
+            const float l0 = (kOtcKs < 16 ? __uint_as_float(o[0]) + p0 : __uint_as_float(o[0])) + wo[2 * kHidden + 0];
+            const float l1 = (kOtcKs < 16 ? __uint_as_float(o[1]) + p1 : __uint_as_float(o[1])) + wo[2 * kHidden + 1];
             if (logits) {
               logits[io * 2 + 0] = l0;
               logits[io * 2 + 1] = l1;
@@ -1387,7 +1469,7 @@ cudaError_t launch_t(const void *in, const TileSched &ts, int nh_layout, uint8_t
     if (e != cudaSuccess) return e;
     attr_set[dev & 63].store(true, std::memory_order_release);
   }
-  mlp_tc_kernel<PREC, IN_KIND, OTC><<<grid, kThreads, L.total + kTraceBytes, s>>>(in, ts, nh_layout,
+  mlp_tc_kernel<PREC, IN_KIND, OTC><<<grid, threads_of<OTC>(), L.total + kTraceBytes, s>>>(in, ts, nh_layout,
                                                                                  dec, logits);
   return cudaGetLastError();
 }

@@ -17,6 +17,7 @@ KIND = {1: "XFULL", 2: "TEMPTY", 3: "HREADY", 4: "COMMIT", 5: "DFULL", 6: "CHUNK
         13: "FENCE", 14: "TOP", 15: "SCHED", 16: "WREADY", 17: "MMA0", 18: "CX", 19: "O_HDONE",
         20: "O_COMMIT", 21: "E_HDONE", 22: "E_DOUT", 23: "E_TEMPTY"}
 STREAM = ({0: "mma", 1: "dig0", 2: "dig1", 3: "epi3"} if os.environ.get("LAKE_TRACE_DIG") else
+          {0: "mma", 1: "g0pl", 2: "g1pl", 3: "dig"} if os.environ.get("LAKE_TRACE_OTC") else
           {0: "mma", 1: "e3r1", 2: "e3r2", 3: "e7r1"} if os.environ.get("LAKE_TRACE_PAIR") else {0: "q0w4", 1: "q1w5", 2: "q2w6", 3: "q3w3"} if os.environ.get("LAKE_TRACE_QUAD") else {0: "mma", 1: "epi4", 2: "epi11", 3: "dig"})
 CAP = int(os.environ.get("LAKE_TRACE_CAP", 1 << 16))  # 512 for the SMEM-log build (-DLAKE_TRACE_SMEM)
 
