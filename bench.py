@@ -39,6 +39,7 @@ ARCH_NAME = {0: "NN (31-256-2)", 1: "NN+1 (31-256-256-2)", 2: "NN+2 (31-256-256-
 ARCH_FLOPS = {0: 2 * (31 * 256 + 256 * 2), 1: 2 * (31 * 256 + 256 * 256 + 256 * 2),
               2: 2 * (31 * 256 + 2 * 256 * 256 + 256 * 2)}
 RAW_BYTES = 36
+NN_OTC_CYCLES_PER_TILE = 2 * 128.1 + 16 * 62.1  # NN fp16/bf16 tile on the tensor pipe (DESIGN 6.3)
 L2_BYTES = 126 * 1024 * 1024
 THROTTLE_BAD = ("hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown")
 
@@ -784,10 +785,20 @@ def run_report(args):
                 ms = timed(lambda: lake.infer(big, fl, 1 << 24, 0, dbig, None, stream))
                 tflops = ARCH_FLOPS[0] * (1 << 24) / (ms / 1e3) / 1e12
                 gbs = (RAW_BYTES + 1) * (1 << 24) / (ms / 1e3) / 1e9
-                rows.append(dict(config="C4-single", arch="NN", path=prec, n=1 << 24, ms=round(ms, 4),
-                                 inferences_per_s=round((1 << 24) / (ms / 1e3), 1),
-                                 tflops=round(tflops, 2), frac_of_peak=round(tflops / peak_of(prec), 4),
-                                 peak=peak_label(prec), hbm_gb_s=round(gbs, 1)))
+                row = dict(config="C4-single", arch="NN", path=prec, n=1 << 24, ms=round(ms, 4),
+                           inferences_per_s=round((1 << 24) / (ms / 1e3), 1),
+                           tflops=round(tflops, 2), frac_of_peak=round(tflops / peak_of(prec), 4),
+                           peak=peak_label(prec), hbm_gb_s=round(gbs, 1))
+                if prec in ("f16", "bf16"):
+                    # NN's tensor-core bound is the MMA instruction rate, not FLOPs: per 256-row
+                    # tile 2 layer-0 MMAs (N=256, 128.1 cycles) + 16 output-layer MMAs (N=16,
+                    # 62.1 cycles: the per-instruction floor, scripts/microbench/umma_dep.cu),
+                    # tiles spread over 74 CTA pairs, at the SM max clock
+                    tiles_per_pair = ((1 << 24) // 256 + 73) // 74
+                    bound_ms = NN_OTC_CYCLES_PER_TILE * tiles_per_pair / (peaks.get("sm_max_mhz", 1965.0) * 1e3)
+                    row.update(mma_instr_bound_ms=round(bound_ms, 4),
+                               frac_of_mma_instr_bound=round(bound_ms / ms, 4))
+                rows.append(row)
                 log(json.dumps(rows[-1]))
             del big, dbig
         for m in w["models"]:

@@ -18,6 +18,7 @@
 
 #include "digitize.cuh"
 #include "lake_internal.h"
+#include "lake_ptx.cuh"
 
 namespace lake {
 namespace {
@@ -423,6 +424,164 @@ group_scatter_pack(const IdT *__restrict__ ids, int64_t n, WsHeader *h, int32_t 
   }
 }
 
+// The same scatter + packing for raw records with 16-B-aligned records and ids, fed by bulk
+// copies (cp.async.bulk, TMA engine) instead of per-warp loads: one block of 512 threads per
+// SM streams its chunks' records and ids as 1,024-I/O sub-chunks (36 KB + ids) through a
+// kTmaStages-deep shared-memory ring, so DRAM reads stay in flight across the per-chunk
+// scan / reservation / write-out phases (the load-based kernel above exposed a DRAM latency
+// per iteration: long-scoreboard stalls, 50% of HBM peak). Sorting, reservation and the
+// per-model runs are those of group_scatter_pack.
+#ifndef LAKE_SCATTER_TMA
+#define LAKE_SCATTER_TMA 1
+#endif
+constexpr int kSub = 1024;                     // I/Os per bulk-copied sub-chunk
+constexpr int kTmaStages = 3;
+constexpr int kSubsPerChunk = kChunk / kSub;
+static_assert(kChunk % kSub == 0 && kSub == 2 * kGBlock, "two records per thread per sub-chunk");
+constexpr size_t kSubRawBytes = (size_t)kSub * 36;
+constexpr size_t kSubIdBytes = (size_t)kSub * 4;   // room for int32 ids
+constexpr size_t kTmaSmem = (size_t)kChunk * (16 + 4) + kTmaStages * (kSubRawBytes + kSubIdBytes);
+
+template <typename IdT>
+__global__ void __launch_bounds__(kGBlock, 1)
+group_scatter_pack_tma(const IdT *__restrict__ ids, int64_t n, WsHeader *h,
+                       int32_t *__restrict__ perm, const int32_t *__restrict__ chunk_counts,
+                       const void *__restrict__ in, uint4 *__restrict__ pdig,
+                       int32_t *__restrict__ cursor) {
+  __shared__ int32_t cnt[kBins];
+  __shared__ int32_t loff[kBins];
+  __shared__ int32_t basep[kBins];
+  __shared__ int32_t wsum[kGBlock / 32];
+  __shared__ uint8_t known_s[LAKE_MAX_MODELS];
+  __shared__ __align__(8) uint64_t full[kTmaStages];
+  extern __shared__ __align__(16) uint8_t dyn[];
+  uint4 *srow = reinterpret_cast<uint4 *>(dyn);
+  uint32_t *skey = reinterpret_cast<uint32_t *>(dyn + (size_t)kChunk * 16);
+  uint8_t *ring = dyn + (size_t)kChunk * 20;  // [stage] raw records | ids
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const uint8_t *raw = static_cast<const uint8_t *>(in);
+  const int64_t G = gridDim.x;
+  // sub-chunk q of this block: chunk blockIdx.x + (q / kSubsPerChunk) G, part q % kSubsPerChunk
+  auto sub_base = [&](int64_t q) {
+    return ((int64_t)blockIdx.x + (q / kSubsPerChunk) * G) * kChunk + (q % kSubsPerChunk) * kSub;
+  };
+  auto issue = [&](int64_t q) {  // thread 0: bring sub-chunk q into its ring stage
+    const int64_t sb = sub_base(q);
+    if (sb >= n) return;
+    const int st = (int)(q % kTmaStages);
+    const int64_t c = (n - sb) < kSub ? (n - sb) : kSub;
+    const uint32_t rb = (uint32_t)(c * 36) & ~15u, ib = (uint32_t)(c * sizeof(IdT)) & ~15u;
+    const uint32_t fb = ptx::smem_u32(&full[st]);
+    uint8_t *dst = ring + (size_t)st * (kSubRawBytes + kSubIdBytes);
+    ptx::mbar_arrive_expect_tx(fb, rb + ib);
+    if (rb) ptx::bulk_g2s(ptx::smem_u32(dst), raw + sb * 36, rb, fb);
+    if (ib) ptx::bulk_g2s(ptx::smem_u32(dst + kSubRawBytes), ids + sb, ib, fb);
+  };
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < kTmaStages; ++i) ptx::mbar_init(ptx::smem_u32(&full[i]), 1);
+    ptx::fence_mbar_init();
+  }
+  load_known(h, known_s);
+  __syncthreads();
+  if (threadIdx.x == 0)
+    for (int i = 0; i < kTmaStages; ++i) issue(i);
+  int64_t q = 0;  // next sub-chunk to consume
+  // The chunk histogram loads and the cursor reservations (global atomics with a returned
+  // value) of chunk k+1 are issued during chunk k - loads before its sort phase, atomics
+  // before its write-out - so neither round trip sits between two chunks.
+  const int t = threadIdx.x;
+  int32_t ns[3], nc[3], rv[3];  // next chunk: scan inputs (bins 2t, 2t+1, 1024), counts and
+                                // reserved bases of bins t, t+512, t+1024
+  auto load_next = [&](int64_t b) {
+    const int32_t *cc = chunk_counts + (b / kChunk) * kBins;
+    ns[0] = cc[2 * t];
+    ns[1] = cc[2 * t + 1];
+    ns[2] = t == kGBlock - 1 ? cc[kBins - 1] : 0;
+#pragma unroll
+    for (int i = 0; i < 3; ++i) nc[i] = (t + i * kGBlock < kBins) ? cc[t + i * kGBlock] : 0;
+  };
+  auto reserve_next = [&]() {
+#pragma unroll
+    for (int i = 0; i < 3; ++i)
+      rv[i] = nc[i] ? atomicAdd(&cursor[(t + i * kGBlock) * kCursorStride], nc[i]) : 0;
+  };
+  if ((int64_t)blockIdx.x * kChunk < n) {
+    load_next((int64_t)blockIdx.x * kChunk);
+    reserve_next();
+  }
+  for (int64_t base = (int64_t)blockIdx.x * kChunk; base < n; base += G * kChunk) {
+    const int64_t end = (base + kChunk) < n ? base + kChunk : n;
+    const int64_t nbase = base + G * kChunk;
+    const int b0 = 2 * t;
+    const int32_t c0 = ns[0], c1 = ns[1], c2 = ns[2];
+    int32_t x = c0 + c1 + c2;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int32_t y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane == 31) wsum[w] = x;
+    __syncthreads();
+    int32_t wpre = 0;
+    for (int j = 0; j < w; ++j) wpre += wsum[j];
+    const int32_t excl = wpre + x - (c0 + c1 + c2);
+    loff[b0] = excl;
+    loff[b0 + 1] = excl + c0;
+    if (t == kGBlock - 1) loff[kBins - 1] = excl + c0 + c1;
+#pragma unroll
+    for (int i = 0; i < 3; ++i)
+      if (t + i * kGBlock < kBins) {
+        basep[t + i * kGBlock] = rv[i];
+        cnt[t + i * kGBlock] = 0;
+      }
+    __syncthreads();
+    if (nbase < n) load_next(nbase);
+    // 1) counting sort of the chunk's sub-chunks, each read from its ring stage
+    for (int64_t sb = base; sb < end; sb += kSub, ++q) {
+      const int st = (int)(q % kTmaStages);
+      const int64_t c = (end - sb) < kSub ? (end - sb) : kSub;
+      const uint32_t rb = (uint32_t)(c * 36) & ~15u, ib = (uint32_t)(c * sizeof(IdT)) & ~15u;
+      const uint8_t *sraw = ring + (size_t)st * (kSubRawBytes + kSubIdBytes);
+      const IdT *sid = reinterpret_cast<const IdT *>(sraw + kSubRawBytes);
+      ptx::mbar_wait(ptx::smem_u32(&full[st]), (uint32_t)((q / kTmaStages) & 1));
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        const int r = threadIdx.x + u * kGBlock;
+        if (r >= c) continue;
+        uint32_t rec[9];
+        if ((uint32_t)(r + 1) * 36 <= rb) {  // stride 9 words: conflict-free
+          const uint32_t *src = reinterpret_cast<const uint32_t *>(sraw) + r * 9;
+#pragma unroll
+          for (int f = 0; f < 9; ++f) rec[f] = src[f];
+        } else {  // tail records past the 16-B-multiple prefix
+          const uint32_t *src = reinterpret_cast<const uint32_t *>(raw) + (sb + r) * 9;
+#pragma unroll
+          for (int f = 0; f < 9; ++f) rec[f] = __ldg(src + f);
+        }
+        const int32_t id = (uint32_t)(r + 1) * sizeof(IdT) <= ib ? (int32_t)sid[r] : (int32_t)__ldg(ids + sb + r);
+        const uint4 pk = pack_record(rec);
+        const int32_t m = bin_of(known_s, id);
+        const int32_t lp = loff[m] + atomicAdd(&cnt[m], 1);
+        srow[lp] = pk;
+        skey[lp] = ((uint32_t)m << 16) | (uint32_t)(sb + r - base);
+      }
+      __syncthreads();  // stage st fully read
+      if (threadIdx.x == 0) issue(q + kTmaStages);
+    }
+    if (nbase < n) reserve_next();
+    // 2) contiguous per-model runs out
+    const int nk = (int)(end - base);
+    for (int k = threadIdx.x; k < nk; k += kGBlock) {
+      const uint32_t e = skey[k];
+      const int m = (int)(e >> 16);
+      const int32_t pos = basep[m] + (k - loff[m]);
+      perm[pos] = (int32_t)(base + (e & 0xFFFFu));
+      if (m < LAKE_MAX_MODELS) pdig[pos] = srow[k];
+    }
+    __syncthreads();
+  }
+}
+
 __device__ __forceinline__ int find_model(const int32_t *off, int32_t t) {
   int lo = 0, hi = LAKE_MAX_MODELS;  // off[lo] <= t < off[hi]
   while (hi - lo > 1) {
@@ -559,7 +718,17 @@ cudaError_t launch_group(int64_t n, const void *model_ids, int id_kind, const De
     if (!in)
       group_scatter<IdT, -1><<<grid, kGBlock, 0, s>>>(ids, n, p.h, p.perm, p.cc, nullptr, nullptr,
                                                       p.cursor);
-    else if (in_kind == LAKE_IN_RAW)
+    else if (in_kind == LAKE_IN_RAW && LAKE_SCATTER_TMA &&
+             (reinterpret_cast<uintptr_t>(in) & 15) == 0 && (reinterpret_cast<uintptr_t>(ids) & 15) == 0) {
+      auto kern = group_scatter_pack_tma<IdT>;
+      static std::atomic<bool> attr_t[64];
+      if (!attr_t[dev & 63].load(std::memory_order_acquire)) {
+        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTmaSmem);
+        attr_t[dev & 63].store(true, std::memory_order_release);
+      }
+      const int tgrid = (int)(chunks < sms ? chunks : sms);
+      kern<<<tgrid, kGBlock, kTmaSmem, s>>>(ids, n, p.h, p.perm, p.cc, in, p.pdig, p.cursor);
+    } else if (in_kind == LAKE_IN_RAW)
       scatter_pack(group_scatter_pack<IdT, LAKE_IN_RAW>, ids);
     else
       scatter_pack(group_scatter_pack<IdT, LAKE_IN_DIGITS>, ids);
