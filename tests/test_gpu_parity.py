@@ -291,6 +291,39 @@ def test_multi_order_invariance(multi_models):
     assert np.array_equal(lg[p].view(np.uint32), lg2.view(np.uint32))
 
 
+@pytest.mark.parametrize("n", [30001, 4096 * 3 + 1023])
+@pytest.mark.parametrize("prec", [lake.LAKE_PREC_F16, lake.LAKE_PREC_FP32])
+def test_multi_misaligned_inputs_same_bits(multi_models, n, prec):
+    """Both grouping scatters give the same results: 16-B-aligned raw records and ids take
+    the bulk-copy-fed scatter (sub-chunk tails past the 16-B prefix read from global), a
+    misaligned record or id array the load-based one; ragged chunk and sub-chunk tails."""
+    import torch
+    raw, mids = inputs.multi_device_trace(n, 3, seed_base=700, rerate=3.0)
+    ids = np.array(list(multi_models))[mids].astype(np.int32)
+    flags = lake.LAKE_IN_RAW | prec
+    lg, dec, unk = run_multi(raw, ids, flags)
+    assert unk == 0
+    dev = "cuda:0"
+    rbuf = torch.zeros(n * 9 + 1, dtype=torch.int32, device=dev)
+    rbuf[1:].copy_(torch.from_numpy(np.ascontiguousarray(raw).view(np.int32).reshape(-1)).to(dev))
+    ibuf = torch.zeros(n + 1, dtype=torch.int32, device=dev)
+    ibuf[1:].copy_(torch.from_numpy(ids).to(dev))
+    for x, d_ids in ((rbuf[1:], cuda(ids)), (cuda(raw), ibuf[1:]), (rbuf[1:], ibuf[1:])):
+        assert x.data_ptr() % 16 != 0 or d_ids.data_ptr() % 16 != 0
+        d = torch.full((n,), 7, dtype=torch.uint8, device=dev)
+        l = torch.full((n, 2), 12345.0, dtype=torch.float32, device=dev)
+        wsb = lake.workspace_bytes(n)
+        ws = torch.empty(wsb, dtype=torch.uint8, device=dev)
+        lake.infer_multi(x, flags, n, d_ids, d, l, ws, wsb)
+        torch.cuda.synchronize()
+        assert np.array_equal(d.cpu().numpy(), dec)
+        assert np.array_equal(l.cpu().numpy().view(np.uint32), lg.view(np.uint32))
+    if prec == lake.LAKE_PREC_FP32:
+        rlg, rdec = oracle.infer_multi_raw(
+            {m: (a, inputs.weights(a, m)) for m, a in multi_models.items()}, raw, ids, nthreads=0)
+        assert np.array_equal(dec, rdec)
+
+
 # ------------------------------------------------------------------------- errors
 def test_error_codes_on_device():
     import torch
