@@ -23,6 +23,7 @@
 #include <atomic>
 
 #include "lake_internal.h"
+#include "lake_ptx.cuh"
 
 namespace lake {
 namespace {
@@ -39,6 +40,9 @@ constexpr int kF32ActBufs = LAKE_F32_ACT_BUFS;
 #define LAKE_F32_CTAS 2  // CTAs per SM (<= 128 registers; A/B: 1 -> 2 CTAs +3% NN+2, +36% NN)
 #endif  // 1: in place (frees SMEM for KC = 64)
 
+#ifndef LAKE_F32_FFMA2
+#define LAKE_F32_FFMA2 0  // 1: hot loop on fma.rn.f32x2 (A/B)
+#endif
 #ifndef LAKE_F32_PF
 #define LAKE_F32_PF 0  // 1: register double buffer of the next k-step (A/B: 6.74 vs 5.76 ms)
 #endif
@@ -171,6 +175,16 @@ mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched t
       for (int i = 0; i < RM; ++i)
 #pragma unroll
         for (int j = 0; j < RN; ++j) acc[i][j] = 0.0f;
+#if LAKE_F32_FFMA2
+      // paired accumulators (columns 2jp, 2jp+1 of row i): one fma.rn.f32x2 does two FMAs,
+      // each rounded exactly as __fmaf_rn (bit-exact); halves the FFMA instruction count of
+      // the issue-bound hot loop
+      uint64_t acc2[RM][RN / 2];
+#pragma unroll
+      for (int i = 0; i < RM; ++i)
+#pragma unroll
+        for (int jp = 0; jp < RN / 2; ++jp) acc2[i][jp] = 0ull;
+#endif
       const int nch = (Kst + KC - 1) / KC;  // layer 0 stages its 32 rows even when KC > 32
       stage_chunk<T>(sm.w[0], wt, Kst < KC ? Kst : KC);
       for (int c = 0; c < nch; ++c) {
@@ -209,7 +223,35 @@ mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched t
             bv[4 * f] = b4.x; bv[4 * f + 1] = b4.y; bv[4 * f + 2] = b4.z; bv[4 * f + 3] = b4.w;
           }
         };
-#if LAKE_F32_PF
+#if LAKE_F32_PF == 2
+        // software-pipelined with two explicit operand sets (no register copies) and no
+        // branches around the loads (a predicated load was sunk below the FFMAs it was meant
+        // to overlap): k-step kk+1's shared loads are issued before kk's FFMAs; the last
+        // iteration's look-ahead load re-reads a valid row and is not used
+        {
+          float a0[RM], b0[RN], a1[RM], b1[RN];
+          load_ops(0, a0, b0);
+          int kk = 0;
+          for (; kk + 1 < kmax; kk += 2) {
+            load_ops(kk + 1, a1, b1);
+#pragma unroll
+            for (int i = 0; i < RM; ++i)
+#pragma unroll
+              for (int j = 0; j < RN; ++j) acc[i][j] = __fmaf_rn(a0[i], b0[j], acc[i][j]);
+            load_ops(kk + 2 < kmax ? kk + 2 : kmax - 1, a0, b0);
+#pragma unroll
+            for (int i = 0; i < RM; ++i)
+#pragma unroll
+              for (int j = 0; j < RN; ++j) acc[i][j] = __fmaf_rn(a1[i], b1[j], acc[i][j]);
+          }
+          if (kk < kmax) {  // odd kmax (layer 0: 31 terms): a0/b0 hold k-step kk
+#pragma unroll
+            for (int i = 0; i < RM; ++i)
+#pragma unroll
+              for (int j = 0; j < RN; ++j) acc[i][j] = __fmaf_rn(a0[i], b0[j], acc[i][j]);
+          }
+        }
+#elif LAKE_F32_PF
         // software-pipelined: k-step kk+1's shared loads are in flight during kk's FFMAs (with
         // two warps per scheduler at RN 16, their latency was the top stall)
         float av[RM], bv[RN];
@@ -232,14 +274,32 @@ mlp_fp32_kernel(const void *__restrict__ in, const __grid_constant__ TileSched t
         for (int kk = 0; kk < kmax; ++kk) {
           float av[RM], bv[RN];
           load_ops(kk, av, bv);
+#if LAKE_F32_FFMA2
+          uint64_t bp[RN / 2];
+#pragma unroll
+          for (int jp = 0; jp < RN / 2; ++jp) bp[jp] = ptx::pack_f32x2(bv[2 * jp], bv[2 * jp + 1]);
+#pragma unroll
+          for (int i = 0; i < RM; ++i) {
+            const uint64_t ap = ptx::pack_f32x2(av[i], av[i]);
+#pragma unroll
+            for (int jp = 0; jp < RN / 2; ++jp) ptx::fma_f32x2(acc2[i][jp], ap, bp[jp]);
+          }
+#else
 #pragma unroll
           for (int i = 0; i < RM; ++i)
 #pragma unroll
             for (int j = 0; j < RN; ++j) acc[i][j] = __fmaf_rn(av[i], bv[j], acc[i][j]);
+#endif
         }
 #endif
         __syncthreads();
       }
+#if LAKE_F32_FFMA2
+#pragma unroll
+      for (int i = 0; i < RM; ++i)
+#pragma unroll
+        for (int jp = 0; jp < RN / 2; ++jp) ptx::unpack_f32x2(acc2[i][jp], acc[i][2 * jp], acc[i][2 * jp + 1]);
+#endif
       // epilogue: z = acc + b (one rounding), ReLU, store transposed
       const float *bias = mp->b[l];
 #pragma unroll
