@@ -303,6 +303,14 @@ __device__ __forceinline__ void tmem_ld_wait() {
 }
 
 // Paired fp32 (fma.rn.f32x2, sm_100): each lane is one IEEE fp32 FMA with a single rounding.
+// The value itself, through a volatile asm: code using the result cannot be hoisted above
+// earlier volatile asm (tcgen05 waits, barriers), so a register loaded early from global
+// memory is first *used* here and its latency overlaps the work in between.
+__device__ __forceinline__ uint32_t opaque_u32(uint32_t x) {
+  uint32_t y;
+  asm volatile("mov.b32 %0, %1;" : "=r"(y) : "r"(x));
+  return y;
+}
 __device__ __forceinline__ uint64_t pack_f32x2(float lo, float hi) {
   uint64_t r;
   asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(lo), "f"(hi));

@@ -1233,7 +1233,10 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           // progresses measured 30% slower: per-chunk group barriers on the packing path.)
           const int pos = (int)(rank * 128 + row);
           const int64_t pp = ti.begin + pos;
-          const int64_t io = (ts.perm && pos < ti.count) ? (int64_t)__ldg(ts.perm + pp) : pp;
+          // the row's output index (multi-model calls): loaded now, first used after the
+          // packing and the output MMA (opaque_u32 below) - its sign extension right after the
+          // load put a DRAM latency in front of the packing (ncu: 14% of stall samples, C4)
+          const uint32_t io_ld = (ts.perm && pos < ti.count) ? (uint32_t)__ldg(ts.perm + pp) : 0u;
           static_assert(!OTC || (kEpiCols == 16 && kChunks == 8 && kEpiPerQ == 2), "OTC packing layout");
           if (ti.model != wcur) {
             // this group's W_out block, rewritten whole (the region held another model's
@@ -1334,6 +1337,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           __syncwarp();
           release_acc(b);
           LAKE_TEV(T_ETEMPTY, it, b, warp);
+          const int64_t io = ts.perm ? (int64_t)(int32_t)ptx::opaque_u32(io_ld) : pp;
           if (hh == 0 && pos < ti.count) {
             if (kOtcKs < 16) {
               p0 += red[row * 2 + 0];  // the quadrant's second warp (written before the barrier)
