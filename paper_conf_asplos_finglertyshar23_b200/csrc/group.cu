@@ -544,26 +544,40 @@ group_scatter_pack_tma(const IdT *__restrict__ ids, int64_t n, WsHeader *h,
       const uint8_t *sraw = ring + (size_t)st * (kSubRawBytes + kSubIdBytes);
       const IdT *sid = reinterpret_cast<const IdT *>(sraw + kSubRawBytes);
       ptx::mbar_wait(ptx::smem_u32(&full[st]), (uint32_t)((q / kTmaStages) & 1));
-#pragma unroll
-      for (int u = 0; u < 2; ++u) {
-        const int r = threadIdx.x + u * kGBlock;
-        if (r >= c) continue;
-        uint32_t rec[9];
-        if ((uint32_t)(r + 1) * 36 <= rb) {  // stride 9 words: conflict-free
-          const uint32_t *src = reinterpret_cast<const uint32_t *>(sraw) + r * 9;
-#pragma unroll
-          for (int f = 0; f < 9; ++f) rec[f] = src[f];
-        } else {  // tail records past the 16-B-multiple prefix
-          const uint32_t *src = reinterpret_cast<const uint32_t *>(raw) + (sb + r) * 9;
-#pragma unroll
-          for (int f = 0; f < 9; ++f) rec[f] = __ldg(src + f);
-        }
-        const int32_t id = (uint32_t)(r + 1) * sizeof(IdT) <= ib ? (int32_t)sid[r] : (int32_t)__ldg(ids + sb + r);
+      auto sort_one = [&](int r, const uint32_t (&rec)[9], int32_t id) {
         const uint4 pk = pack_record(rec);
         const int32_t m = bin_of(known_s, id);
         const int32_t lp = loff[m] + atomicAdd(&cnt[m], 1);
         srow[lp] = pk;
         skey[lp] = ((uint32_t)m << 16) | (uint32_t)(sb + r - base);
+      };
+      if (c == kSub) {  // full sub-chunk (all but the call's last): shared memory only
+#pragma unroll
+        for (int u = 0; u < 2; ++u) {
+          const int r = threadIdx.x + u * kGBlock;
+          uint32_t rec[9];
+          const uint32_t *src = reinterpret_cast<const uint32_t *>(sraw) + r * 9;  // conflict-free
+#pragma unroll
+          for (int f = 0; f < 9; ++f) rec[f] = src[f];
+          sort_one(r, rec, (int32_t)sid[r]);
+        }
+      } else {
+#pragma unroll
+        for (int u = 0; u < 2; ++u) {
+          const int r = threadIdx.x + u * kGBlock;
+          if (r >= c) continue;
+          uint32_t rec[9];
+          if ((uint32_t)(r + 1) * 36 <= rb) {
+            const uint32_t *src = reinterpret_cast<const uint32_t *>(sraw) + r * 9;
+#pragma unroll
+            for (int f = 0; f < 9; ++f) rec[f] = src[f];
+          } else {  // tail records past the 16-B-multiple prefix
+            const uint32_t *src = reinterpret_cast<const uint32_t *>(raw) + (sb + r) * 9;
+#pragma unroll
+            for (int f = 0; f < 9; ++f) rec[f] = __ldg(src + f);
+          }
+          sort_one(r, rec, (uint32_t)(r + 1) * sizeof(IdT) <= ib ? (int32_t)sid[r] : (int32_t)__ldg(ids + sb + r));
+        }
       }
       __syncthreads();  // stage st fully read
       if (threadIdx.x == 0) issue(q + kTmaStages);
