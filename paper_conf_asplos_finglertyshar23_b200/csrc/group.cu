@@ -137,6 +137,21 @@ group_hist(const IdT *__restrict__ ids, int64_t n, WsHeader *h,
     for (int i = threadIdx.x; i <= LAKE_MAX_MODELS; i += kGBlock) cnt[i] = 0;
     __syncthreads();
     const int64_t end = (base + kChunk) < n ? base + kChunk : n;
+    if (sizeof(IdT) == 4 && end - base == kChunk && (reinterpret_cast<uintptr_t>(ids) & 15) == 0) {
+      // full chunk of 16-B-aligned int32 ids: 16-B loads, all of the thread's in flight at once
+      constexpr int V = kChunk / (4 * kGBlock);
+      int4 v[V];
+#pragma unroll
+      for (int u = 0; u < V; ++u)
+        v[u] = __ldg(reinterpret_cast<const int4 *>(ids + base) + threadIdx.x + u * kGBlock);
+#pragma unroll
+      for (int u = 0; u < V; ++u) {
+        atomicAdd(&cnt[bin_of(known_s, v[u].x)], 1);
+        atomicAdd(&cnt[bin_of(known_s, v[u].y)], 1);
+        atomicAdd(&cnt[bin_of(known_s, v[u].z)], 1);
+        atomicAdd(&cnt[bin_of(known_s, v[u].w)], 1);
+      }
+    } else
     for (int64_t i0 = base + threadIdx.x; i0 < end; i0 += 4 * kGBlock) {
       int32_t idv[4];  // four loads in flight per thread
 #pragma unroll
