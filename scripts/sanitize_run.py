@@ -76,3 +76,17 @@ if os.environ.get("SANITIZE_SERVER", "1") == "1":
         srv.infer(np.ascontiguousarray(raw[:64]), 64, hd)
 torch.cuda.synchronize()
 print("sanitize run ok")
+if os.environ.get("LAKE_SAN_BIG"):
+    # more 4,096-I/O chunks than scatter blocks (one per SM): every block streams several
+    # chunks through its bulk-copy ring (next-chunk histogram loads and reservations)
+    nb = 148 * 4096 * 2 + 777
+    rawb = inputs.edge_raw(nb, seed=2)
+    xb = torch.from_numpy(rawb.view(np.int32)).to(dev)
+    idsb = torch.from_numpy(np.random.default_rng(1).integers(1, 4, nb).astype(np.int32)).to(dev)
+    decb = torch.empty(nb, dtype=torch.uint8, device=dev)
+    wsbb = lake.workspace_bytes(nb)
+    wsb_t = torch.empty(wsbb, dtype=torch.uint8, device=dev)
+    lake.multi_group(nb, idsb, wsb_t, wsbb)
+    lake.infer_multi(xb, lake.LAKE_IN_RAW | lake.LAKE_PREC_F16, nb, idsb, decb, None, wsb_t, wsbb)
+    torch.cuda.synchronize()
+    print("big multi ok")

@@ -324,6 +324,23 @@ def test_multi_misaligned_inputs_same_bits(multi_models, n, prec):
         assert np.array_equal(dec, rdec)
 
 
+def test_multi_many_chunks_per_block_equals_per_model(multi_models):
+    """More 4,096-I/O chunks than grouping-scatter blocks (one per SM): each block streams
+    several chunks through its bulk-copy ring; every row of infer_multi equals the per-model
+    call bit for bit (fp16), so no row is lost, duplicated or paired with another's index."""
+    n = 148 * 4096 * 2 + 777
+    raw, mids = inputs.multi_device_trace(n, 3, seed_base=800, rerate=3.0)
+    ids = np.array(list(multi_models))[mids].astype(np.int32)
+    flags = lake.LAKE_IN_RAW | lake.LAKE_PREC_F16
+    lg, dec, unk = run_multi(raw, ids, flags)
+    assert unk == 0
+    for m in multi_models:
+        idx = np.nonzero(ids == m)[0]
+        slg, sdec = run_infer(m, raw[idx], flags)
+        assert np.array_equal(dec[idx], sdec)
+        assert np.array_equal(lg[idx].view(np.uint32), slg.view(np.uint32))
+
+
 # ------------------------------------------------------------------------- errors
 def test_error_codes_on_device():
     import torch
