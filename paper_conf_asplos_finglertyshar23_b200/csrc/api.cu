@@ -651,7 +651,10 @@ int lake_linnos_multi_status(const void *workspace, size_t ws_bytes, int64_t *n_
 // stream), two staging slots, so the PCIe transfers of neighbouring chunks overlap compute.
 namespace lake {
 namespace {
-constexpr int64_t kHostChunk = 1 << 20;
+#ifndef LAKE_HOST_CHUNK_LOG2
+#define LAKE_HOST_CHUNK_LOG2 20
+#endif
+constexpr int64_t kHostChunk = (int64_t)1 << LAKE_HOST_CHUNK_LOG2;  // I/Os per pipelined chunk
 constexpr int64_t kZeroCopyMax = 1 << 14;
 
 // Device-accessible alias of a pinned, mapped host pointer (UVA), or nullptr.
