@@ -186,7 +186,9 @@ size_t lake_linnos_workspace_bytes(int64_t n);
  * of the type flags & LAKE_IDS_MASK selects: int32_t by default, uint16_t, uint8_t).
  * Groups I/Os by model on the device (histogram, scan, scatter of indices; the order inside
  * a model's group is not preserved and does not affect any result; tensor-core paths also
- * write each I/O's digits as a 16-byte packed row at its grouped position), then
+ * write each I/O's digits as a 16-byte packed row at its grouped position; with 16-B
+ * aligned raw records and ids that pass streams them through shared memory with bulk
+ * copies, otherwise it loads them per warp - same results either way), then
  * runs the fused kernel over model-homogeneous tiles and scatters results back to the
  * caller's order. Results equal per-model lake_linnos_infer calls bit for bit.
  * workspace: device buffer of at least lake_linnos_workspace_bytes(n) bytes (else
