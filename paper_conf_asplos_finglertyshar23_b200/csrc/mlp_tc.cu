@@ -240,9 +240,9 @@ __host__ __device__ constexpr Layout tc_layout(int nh_layout, int prec) {
   // group 0's own copy of the output-layer parameters and partial sums: with two epilogue
   // groups, NN tiles (a single layer) are drained by the group of their accumulator buffer
   L.prm0 = L.red + kRedBytes;
-  L.red0 = L.prm0 + kPrmFloats * 4;
+  L.red0 = L.prm0 + (kEpiGroups == 2 ? kPrmFloats * 4 : 0u);  // (one group: no private copy)
   L.wout = otc_wout(prec);  // behind W0 in the weight region (out_on_tc layouts only)
-  L.bar = L.red0 + kRedBytes;
+  L.bar = L.red0 + (kEpiGroups == 2 ? kRedBytes : 0u);
   L.total = L.bar + 512;
   return L;
 }
