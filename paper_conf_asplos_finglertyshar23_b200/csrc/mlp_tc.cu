@@ -110,6 +110,18 @@ constexpr uint32_t kEpiPerQ = LAKE_EPI_PER_Q;      // epilogue warps per group a
 #define LAKE_EPI_GROUPS 2
 #endif
 constexpr uint32_t kEpiGroups = LAKE_EPI_GROUPS;
+// A/B switch (fp16/bf16, NN+1/NN+2): the last hidden layer as two N = 128 halves, each
+// committed on its own barrier, so the logits epilogue starts on columns 0..127 while the
+// tensor core computes 128..255. With cta_group::2 an N = 128 MMA takes 64 B rows from each
+// CTA, so half h covers features {64h..64h+63} (CTA 0's rows) and {128+64h..} (CTA 1's):
+// accumulator column c holds feature nsplit_feature(c), and W_out is staged in that order.
+#ifndef LAKE_L2_NSPLIT
+#define LAKE_L2_NSPLIT 0
+#endif
+constexpr bool kL2Split = LAKE_L2_NSPLIT != 0;
+__host__ __device__ constexpr uint32_t nsplit_feature(uint32_t c) {
+  return c < 64 ? c : c < 128 ? c + 64 : c < 192 ? c - 64 : c;
+}
 constexpr uint32_t kGroupWarps = 4 * kEpiPerQ;     // warps per epilogue group
 constexpr uint32_t kEpiWarps = kEpiGroups * kGroupWarps;
 #ifndef LAKE_CHUNKS
@@ -258,7 +270,8 @@ enum : uint32_t {
   B_SFULL = B_REMPTY + kTcRingSlots,     // [2] input staging buffer loaded (bulk copy)
   B_HDONE = B_SFULL + 2,                  // [2] out_on_tc: H of buffer b packed (both CTAs)
   B_DOUT = B_HDONE + 2,                   // [2] out_on_tc: output MMA of buffer b done
-  B_COUNT = B_DOUT + 2
+  B_DHALF = B_DOUT + 2,                   // [2] LAKE_L2_NSPLIT: last layer's first half done
+  B_COUNT = B_DHALF + 2
 };
 constexpr uint32_t kTmemSlot = B_COUNT * 8;  // u32 TMEM base address
 static_assert(kTmemSlot + 4 <= 512, "barrier block");
@@ -623,6 +636,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
       ptx::mbar_init(bar(B_XEMPTY + i), 1);      // tcgen05.commit (multicast)
       ptx::mbar_init(bar(B_DFULL + i), 1);       // tcgen05.commit (multicast): H layers
       ptx::mbar_init(bar(B_DFULLX + i), 1);      // tcgen05.commit (multicast): last layer
+      ptx::mbar_init(bar(B_DHALF + i), 1);       // tcgen05.commit (multicast): its first half
 #ifdef LAKE_TEMPTY_AGG
       ptx::mbar_init(bar(B_TEMPTY + i), kGroupWarps + 1);  // leader's group warps + the peer
 #else
@@ -840,9 +854,14 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           // fp16/bf16: the layer's bias first (D = ones x bias-block^T initialises the
           // accumulator; it needs no H, so it is issued before the first chunk wait)
           constexpr uint32_t kAcc = PREC == 2 ? 0u : 1u;
+          const bool split = kL2Split && PREC != 2 && l + 1 == nh;
+          // N = 128 halves: B rows 64..127 of each CTA's image start 8 row groups (1 KB) in
+          constexpr uint32_t kHalfB = (8u * 128u) >> 4;
+          const uint32_t idesc_h = ptx::umma_idesc_f16(PREC, 256, 128);
           if constexpr (PREC != 2)
             if (issuer)
-              ptx::mma_cg2<PREC>(d, onesdesc, wd + (tc_wh_half_bytes(PREC) >> 4), idesc, 0);
+              ptx::mma_cg2<PREC>(d, onesdesc, wd + (tc_wh_half_bytes(PREC) >> 4),
+                                 split ? idesc_h : idesc, 0);
           for (uint32_t kc = 0; kc < kChunks; ++kc) {
 #ifndef LAKE_ABL_NOHREADY  // timing-only ablation: the MMA never waits for H chunks
             ptx::mbar_wait(bar(B_HREADY + kc), (h_phase >> kc) & 1);
@@ -875,12 +894,27 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
               for (uint32_t s = 0; s < kKS; ++s) {
                 const uint32_t ks = kc * kKS + s;
                 if (issuer)
-                  ptx::mma_cg2_ts<PREC>(d, ha + tmem_a_col<PREC>(ks), wd + ks * kStep, idesc,
-                                        ks | kAcc);
+                  ptx::mma_cg2_ts<PREC>(d, ha + tmem_a_col<PREC>(ks), wd + ks * kStep,
+                                        split ? idesc_h : idesc, ks | kAcc);
               }
             }
             __syncwarp();
             LAKE_TEV(T_ISSUED, it, l, kc);
+          }
+          if (split) {
+            // first half (columns 0..127) complete -> the logits group starts on it; the
+            // second half reuses the H chunks already waited for
+            if (issuer) {
+              ptx::mma_commit_cg2(bar(B_DHALF + b), 0x3);
+              ptx::mma_cg2<PREC>(d + 128, onesdesc, wd + (tc_wh_half_bytes(PREC) >> 4) + kHalfB,
+                                 idesc_h, 0);
+            }
+#pragma unroll 1
+            for (uint32_t ks = 0; ks < kKS * kChunks; ++ks)
+              if (issuer)
+                ptx::mma_cg2_ts<PREC>(d + 128, ha + tmem_a_col<PREC>(ks), wd + ks * kStep + kHalfB,
+                                      idesc_h, 1u);
+            __syncwarp();
           }
           if (issuer)
             ptx::mma_commit_cg2(bar((kEpiGroups == 2 && l + 1 == nh ? B_DFULLX : B_DFULL) + b), 0x3);
@@ -1112,6 +1146,7 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
     };
     const DevModel *cur = nullptr;
     uint32_t g = 0, d_phase = 0, dx_phase = 0;  // phase bits per accumulator buffer
+    uint32_t dh_phase = 0;                      // LAKE_L2_NSPLIT: B_DHALF phases
     int64_t it = 0;
     TileInfo nxt;
     if (t_begin < t_end) nxt = tile_info<PREC>(ts, t_begin);
@@ -1131,10 +1166,16 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         }
         if (do_last || (kEpiGroups == 2 && nh == 1)) {
           const float4 *src = reinterpret_cast<const float4 *>(ti.model->b[nh - 1]);
-          for (uint32_t i = et; i < kPrmFloats / 4; i += NG)  // NN: b0 is added by the MMA
+          // (split last layer: b_last and W_out rows staged in accumulator-column order)
+          const bool perm_cols = kL2Split && PREC != 2 && nh >= 2;
+          for (uint32_t i = et; i < kPrmFloats / 4; i += NG) {  // NN: b0 is added by the MMA
+            uint32_t si = i;
+            if (perm_cols && i < 3 * kHidden / 4)
+              si = (i / (kHidden / 4)) * (kHidden / 4) + nsplit_feature(4 * (i % (kHidden / 4))) / 4;
             reinterpret_cast<float4 *>(prm)[i] = (nh == 1 && i < kHidden / 4)
                                                      ? make_float4(0.0f, 0.0f, 0.0f, 0.0f)
-                                                     : __ldg(src + i);
+                                                     : __ldg(src + si);
+          }
         }
         ptx::named_bar_sync(2 + gy, NG);
         cur = ti.model;
@@ -1147,8 +1188,10 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
         if (nn2 ? gy != b : !(last ? do_last : do_h)) continue;
         {
           const bool x = kEpiGroups == 2 && (nn2 ? b == 1 : last);
-          const uint32_t wb = x ? bar(B_DFULLX + b) : bar(B_DFULL + b);
-          const uint32_t wp = ((x ? dx_phase : d_phase) >> b) & 1;
+          // split last layer: start on its first half (B_DHALF); B_DFULLX is waited mid-way
+          const bool hx = kL2Split && PREC != 2 && last && nh >= 2;
+          const uint32_t wb = hx ? bar(B_DHALF + b) : x ? bar(B_DFULLX + b) : bar(B_DFULL + b);
+          const uint32_t wp = ((hx ? dh_phase : x ? dx_phase : d_phase) >> b) & 1;
 #ifndef LAKE_EPI_POLL_ALL
           // One warp of the group polls the mbarrier (warp lw = 1: not on the MMA warp's SM
           // sub-partition), the others wait on the group's named barrier. Eight warps spinning
@@ -1159,7 +1202,8 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
 #else
           ptx::mbar_wait(wb, wp);
 #endif
-          if (x) dx_phase ^= (1u << b);
+          if (hx) dh_phase ^= (1u << b);
+          else if (x) dx_phase ^= (1u << b);
           else d_phase ^= (1u << b);
         }
         LAKE_TEV(T_DFULL, it, l, warp);
@@ -1361,16 +1405,27 @@ mlp_tc_kernel(const void *__restrict__ in, const __grid_constant__ TileSched ts,
           const int64_t pp = ti.begin + pos;
           const int64_t io = (ts.perm && pos < ti.count) ? (int64_t)__ldg(ts.perm + pp) : pp;
           float p[4] = {0.0f, 0.0f, 0.0f, 0.0f};
+          const bool hsplit = kL2Split && PREC != 2 && nh >= 2;  // columns 128.. land later
 #pragma unroll kEpiUnroll
           for (uint32_t j = 0; j < kWarpChunks; ++j) {
             const uint32_t col0 = col_of(j);
             if constexpr (kPrefetch) {
-              if (j + 1 < kWarpChunks) {
+              const bool mid = hsplit && j + 1 == kWarpChunks / 2;  // next chunk: 2nd half
+              if (j + 1 < kWarpChunks && !mid) {
                 if (j & 1) ptx::tmem_ld_cols<W>(tbase + col_of(j + 1), ra);
                 else ptx::tmem_ld_cols<W>(tbase + col_of(j + 1), rb);
               }
               if (j & 1) EPI_L(rb);
               else EPI_L(ra);
+              if (mid) {
+                // second half of the last layer: wait for the whole accumulator, then load
+                if (lw == 1) ptx::mbar_wait(bar(B_DFULLX + b), (dx_phase >> b) & 1);
+                ptx::named_bar_sync(2 + gy, NG);
+                dx_phase ^= (1u << b);
+                ptx::tc_fence_after();
+                if (j & 1) ptx::tmem_ld_cols<W>(tbase + col_of(j + 1), ra);
+                else ptx::tmem_ld_cols<W>(tbase + col_of(j + 1), rb);
+              }
               if (j + 1 < kWarpChunks) ptx::tmem_ld_wait();
             } else {
               if (j > 0) {
