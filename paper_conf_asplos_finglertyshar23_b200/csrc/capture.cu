@@ -22,24 +22,72 @@ namespace {
 constexpr int kTimeBits = 47;
 constexpr uint64_t kTimeMask = (1ull << kTimeBits) - 1;
 
-__device__ __forceinline__ uint64_t ckey(int32_t dev, int64_t t) {
-  return ((uint64_t)(uint32_t)(dev & 0xFFFF) << kTimeBits) | ((uint64_t)t & kTimeMask);
+// Compact sort keys: (device << tb) | (time - tmin), with tb the bit width of the trace's
+// time span and only as many 8-bit radix passes as the key's significant bits need (if that
+// is odd, the sorted data ends in the _alt buffers and the consumers pick by its parity):
+// the same order as the full 63-bit (device << 47 | time) key, in 4-6 passes instead of 8
+// for traces spanning seconds.
+struct KeyParams {
+  unsigned long long tmin, tmax;  // over arrivals and completions (47-bit times)
+  unsigned int dmax;              // largest device id (16 bits)
+  int32_t tb;                     // time bits of the key
+  int32_t npasses;                // radix passes of both sorts
+};
+
+__device__ __forceinline__ uint64_t ckey(const KeyParams &p, int32_t dev, int64_t t) {
+  return ((uint64_t)(uint32_t)(dev & 0xFFFF) << p.tb) | (((uint64_t)t & kTimeMask) - p.tmin);
+}
+
+__global__ void key_range(const int64_t *__restrict__ a, const int64_t *__restrict__ c,
+                          const int32_t *__restrict__ dev, int64_t n, KeyParams *p) {
+  unsigned long long lo = ~0ull, hi = 0;
+  unsigned int dm = 0;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const unsigned long long ta = (uint64_t)a[i] & kTimeMask, tc = (uint64_t)c[i] & kTimeMask;
+    lo = min(lo, min(ta, tc));
+    hi = max(hi, max(ta, tc));
+    if (dev) dm = max(dm, (unsigned int)(dev[i] & 0xFFFF));
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    lo = min(lo, __shfl_xor_sync(0xffffffffu, lo, o));
+    hi = max(hi, __shfl_xor_sync(0xffffffffu, hi, o));
+    dm = max(dm, __shfl_xor_sync(0xffffffffu, dm, o));
+  }
+  if ((threadIdx.x & 31) == 0) {
+    atomicMin(&p->tmin, lo);
+    atomicMax(&p->tmax, hi);
+    atomicMax(&p->dmax, dm);
+  }
+}
+
+__global__ void key_params(KeyParams *p) {
+  const uint64_t span = p->tmax >= p->tmin ? p->tmax - p->tmin : 0;
+  const int tb = span ? 64 - __clzll((long long)span) : 1;
+  const int db = p->dmax ? 32 - __clz((int)p->dmax) : 0;
+  const int passes = (tb + db + 7) / 8;
+  p->tb = tb;
+  p->npasses = passes;  // odd: the sorted data ends in the _alt buffers (consumers check)
 }
 
 __global__ void make_keys(const int64_t *__restrict__ a, const int64_t *__restrict__ c,
                           const int32_t *__restrict__ dev, int64_t n, uint64_t *ka, uint64_t *kc,
-                          int32_t *ic, int32_t *ia) {
+                          int32_t *ic, int32_t *ia, const KeyParams *__restrict__ pp) {
+  const KeyParams p = *pp;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
        i += (int64_t)gridDim.x * blockDim.x) {
     const int32_t d = dev ? dev[i] : 0;
-    ka[i] = ckey(d, a[i]);
-    kc[i] = ckey(d, c[i]);
+    ka[i] = ckey(p, d, a[i]);
+    kc[i] = ckey(p, d, c[i]);
     ic[i] = (int32_t)i;
     ia[i] = (int32_t)i;
   }
 }
 
-__global__ void invert(const int32_t *__restrict__ idx, int64_t n, int32_t *rank) {
+__global__ void invert(const int32_t *__restrict__ idx0, const int32_t *__restrict__ idx1,
+                       int64_t n, int32_t *rank, const KeyParams *__restrict__ pp) {
+  const int32_t *idx = (pp->npasses & 1) ? idx1 : idx0;  // where the sort left its result
   for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < n;
        p += (int64_t)gridDim.x * blockDim.x)
     rank[idx[p]] = (int32_t)p;
@@ -59,23 +107,29 @@ __device__ __forceinline__ int64_t bsearch(const uint64_t *__restrict__ keys, in
 }
 
 __global__ void pending_count(const int64_t *__restrict__ a, const int32_t *__restrict__ dev,
-                              int64_t n, const uint64_t *__restrict__ kc_sorted,
+                              int64_t n, const uint64_t *__restrict__ kc0,
+                              const uint64_t *__restrict__ kc1,
                               const int32_t *__restrict__ rank_a, int32_t *q,
-                              int64_t *ub_out) {
+                              int64_t *ub_out, const KeyParams *__restrict__ pp) {
+  const KeyParams p = *pp;
+  const uint64_t *kc_sorted = (p.npasses & 1) ? kc1 : kc0;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
        i += (int64_t)gridDim.x * blockDim.x) {
     const int32_t d = dev ? dev[i] : 0;
-    const int64_t start = bsearch(kc_sorted, n, ckey(d, 0), false);  // device segment start
-    const int64_t ub = bsearch(kc_sorted, n, ckey(d, a[i]), true);   // completions <= a_i
+    // device segment start: the smallest key of device d (time offset 0)
+    const int64_t start = bsearch(kc_sorted, n, (uint64_t)(uint32_t)(d & 0xFFFF) << p.tb, false);
+    const int64_t ub = bsearch(kc_sorted, n, ckey(p, d, a[i]), true);   // completions <= a_i
     q[i] = (int32_t)((rank_a[i] - start + 1) - (ub - start));
     ub_out[i] = ((int64_t)start << 32) | (ub - start);  // (segment start, completed count)
   }
 }
 
 __global__ void history(const int64_t *__restrict__ a, const int64_t *__restrict__ c,
-                        int64_t n, const int32_t *__restrict__ idx_c,
+                        int64_t n, const int32_t *__restrict__ idx_c0,
+                        const int32_t *__restrict__ idx_c1,
                         const int32_t *__restrict__ q, const int64_t *__restrict__ ub_in,
-                        uint32_t *__restrict__ raw) {
+                        uint32_t *__restrict__ raw, const KeyParams *__restrict__ pp) {
+  const int32_t *idx_c = (pp->npasses & 1) ? idx_c1 : idx_c0;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
        i += (int64_t)gridDim.x * blockDim.x) {
     const int64_t start = ub_in[i] >> 32, cnt = ub_in[i] & 0xFFFFFFFFll;
@@ -101,7 +155,7 @@ __global__ void history(const int64_t *__restrict__ a, const int64_t *__restrict
 size_t a256(size_t x) { return (x + 255) & ~(size_t)255; }
 
 struct CapLayout {
-  size_t ka, kc, ka2, kc2, iota, ia, ic, rank, q, ub, sort, total;
+  size_t ka, kc, ka2, kc2, iota, ia, ia2, ic, rank, q, ub, sort, kp, total;
 };
 
 CapLayout cap_layout(int64_t n, size_t sort_bytes) {
@@ -113,11 +167,13 @@ CapLayout cap_layout(int64_t n, size_t sort_bytes) {
   L.kc2 = o; o += a256(n * 8);
   L.iota = o; o += a256(n * 4);
   L.ia = o; o += a256(n * 4);
+  L.ia2 = o; o += a256(n * 4);  // the arrival sort's own alternate (odd pass counts)
   L.ic = o; o += a256(n * 4);
   L.rank = o; o += a256(n * 4);
   L.q = o; o += a256(n * 4);
   L.ub = o; o += a256(n * 8);
   L.sort = o; o += a256(sort_bytes);
+  L.kp = o; o += a256(sizeof(KeyParams));
   L.total = o;
   return L;
 }
@@ -138,26 +194,36 @@ cudaError_t launch_capture(const int64_t *a, const int64_t *c, const int32_t *de
   const int threads = 256;
   const int grid = (int)((n + threads - 1) / threads < 148 * 16 ? (n + threads - 1) / threads
                                                                 : 148 * 16);
-  make_keys<<<grid, threads, 0, s>>>(a, c, dev, n, U64(L.ka), U64(L.kc), I32(L.ic), I32(L.ia));
-  // (device, completion, index) and (device, arrival, index) orders; 8 passes of 8 bits,
-  // so the results land back in kc / ic and ka / ia
+  KeyParams *kp = reinterpret_cast<KeyParams *>(b + L.kp);
+  if (n <= 0) return cudaSuccess;
+  // key range: tmin = all ones, tmax = dmax = 0, then atomics
+  cudaError_t e = cudaMemsetAsync(kp, 0, sizeof(KeyParams), s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(&kp->tmin, 0xFF, sizeof(kp->tmin), s);
+  if (e != cudaSuccess) return e;
+  key_range<<<grid, threads, 0, s>>>(a, c, dev, n, kp);
+  key_params<<<1, 1, 0, s>>>(kp);
+  make_keys<<<grid, threads, 0, s>>>(a, c, dev, n, U64(L.ka), U64(L.kc), I32(L.ic), I32(L.ia), kp);
+  // (device, completion, index) and (device, arrival, index) orders; up to 8 passes of 8
+  // bits, the device skipping the top ones the compact keys do not need (an even count), so
+  // the results land back in kc / ic and ka / ia
   bool alt_c = false, alt_a = false;
-  cudaError_t e = radix_sort_pairs(U64(L.kc), U64(L.kc2), I32(L.ic), I32(L.iota), n,
-                                   kTimeBits + 16, b + L.sort, s, &alt_c);
+  const int32_t *np = &kp->npasses;
+  e = radix_sort_pairs(U64(L.kc), U64(L.kc2), I32(L.ic), I32(L.iota), n, kTimeBits + 16,
+                       b + L.sort, s, &alt_c, np);
   if (e != cudaSuccess) return e;
-  e = radix_sort_pairs(U64(L.ka), U64(L.ka2), I32(L.ia), I32(L.iota), n, kTimeBits + 16,
-                       b + L.sort, s, &alt_a);
+  e = radix_sort_pairs(U64(L.ka), U64(L.ka2), I32(L.ia), I32(L.ia2), n, kTimeBits + 16,
+                       b + L.sort, s, &alt_a, np);
   if (e != cudaSuccess) return e;
-  const uint64_t *kc_sorted = alt_c ? U64(L.kc2) : U64(L.kc);
-  const int32_t *idx_c = alt_c ? I32(L.iota) : I32(L.ic);
-  const int32_t *idx_a = alt_a ? I32(L.iota) : I32(L.ia);
-  static_assert((kTimeBits + 16 + 7) / 8 % 2 == 0, "even pass count: results in place");
-  invert<<<grid, threads, 0, s>>>(idx_a, n, I32(L.rank));
-  pending_count<<<grid, threads, 0, s>>>(a, dev, n, kc_sorted, I32(L.rank), I32(L.q),
-                                         reinterpret_cast<int64_t *>(b + L.ub));
-  history<<<grid, threads, 0, s>>>(a, c, n, idx_c, I32(L.q),
-                                   reinterpret_cast<const int64_t *>(b + L.ub), raw);
-  count_launch(4);
+  // 8 host-side passes always end in kc / ic and ka / ia; the device ran kp->npasses of
+  // them, so the consumers pick the buffers by its parity
+  (void)alt_c;
+  (void)alt_a;
+  invert<<<grid, threads, 0, s>>>(I32(L.ia), I32(L.ia2), n, I32(L.rank), kp);
+  pending_count<<<grid, threads, 0, s>>>(a, dev, n, U64(L.kc), U64(L.kc2), I32(L.rank), I32(L.q),
+                                         reinterpret_cast<int64_t *>(b + L.ub), kp);
+  history<<<grid, threads, 0, s>>>(a, c, n, I32(L.ic), I32(L.iota), I32(L.q),
+                                   reinterpret_cast<const int64_t *>(b + L.ub), raw, kp);
+  count_launch(6);
   return cudaGetLastError();
 }
 

@@ -147,7 +147,8 @@ cudaError_t launch_mlp_tc(const void *in, int in_kind, int prec, const TileSched
 // *in_alt: the result is in the _alt buffers (odd number of 8-bit passes).
 size_t radix_sort_workspace_bytes(int64_t n);
 cudaError_t radix_sort_pairs(uint64_t *keys, uint64_t *keys_alt, int32_t *vals, int32_t *vals_alt,
-                             int64_t n, int bits, void *ws, cudaStream_t s, bool *in_alt);
+                             int64_t n, int bits, void *ws, cudaStream_t s, bool *in_alt,
+                             const int32_t *d_npasses = nullptr);
 // Grouping for infer_multi (group.cu).
 size_t group_workspace_bytes(int64_t n);
 int64_t group_max_tiles(int64_t n, int tile_rows);

@@ -36,7 +36,8 @@ __device__ __forceinline__ uint32_t digit_of(uint64_t k, int shift) {
 
 __global__ void __launch_bounds__(kRsThreads)
 rs_count(const uint64_t *__restrict__ keys, int64_t n, int shift, int32_t *__restrict__ counts,
-         int64_t ntiles) {
+         int64_t ntiles, const int32_t *__restrict__ npasses) {
+  if (npasses && shift / kRsBits >= *npasses) return;  // a skipped (all-zero) digit
   __shared__ int32_t bins[kRsBins];
   bins[threadIdx.x] = 0;
   __syncthreads();
@@ -79,7 +80,9 @@ __device__ __forceinline__ int32_t block_scan1024(int32_t v, int32_t *wsum, int3
 
 // in place: each 4,096-entry block of `a` -> its exclusive scan; bsum[block] = block total
 __global__ void __launch_bounds__(1024)
-rs_scan_blocks(int32_t *__restrict__ a, int64_t m, int32_t *__restrict__ bsum) {
+rs_scan_blocks(int32_t *__restrict__ a, int64_t m, int32_t *__restrict__ bsum, int pass,
+               const int32_t *__restrict__ npasses) {
+  if (npasses && pass >= *npasses) return;
   __shared__ int32_t wsum[32], total;
   const int64_t i0 = (int64_t)blockIdx.x * kRsScanBlock + 4 * threadIdx.x;
   int32_t v[4];
@@ -96,7 +99,9 @@ rs_scan_blocks(int32_t *__restrict__ a, int64_t m, int32_t *__restrict__ bsum) {
 }
 
 // one block: bsum[0..nb) -> exclusive scan, in place (loops over 1,024-entry pieces)
-__global__ void __launch_bounds__(1024) rs_scan_sums(int32_t *__restrict__ bsum, int64_t nb) {
+__global__ void __launch_bounds__(1024) rs_scan_sums(int32_t *__restrict__ bsum, int64_t nb,
+                                                     int pass, const int32_t *__restrict__ npasses) {
+  if (npasses && pass >= *npasses) return;
   __shared__ int32_t wsum[32], total;
   int32_t carry = 0;
   for (int64_t b0 = 0; b0 < nb; b0 += 1024) {
@@ -112,7 +117,9 @@ __global__ void __launch_bounds__(1024) rs_scan_sums(int32_t *__restrict__ bsum,
 __global__ void __launch_bounds__(kRsThreads)
 rs_scatter(const uint64_t *__restrict__ kin, const int32_t *__restrict__ vin, int64_t n, int shift,
            const int32_t *__restrict__ offs, const int32_t *__restrict__ bsum, int64_t ntiles,
-           uint64_t *__restrict__ kout, int32_t *__restrict__ vout) {
+           uint64_t *__restrict__ kout, int32_t *__restrict__ vout,
+           const int32_t *__restrict__ npasses) {
+  if (npasses && shift / kRsBits >= *npasses) return;
   __shared__ uint64_t sk[kRsTile];
   __shared__ int32_t sv[kRsTile];
   __shared__ int32_t whist[kRsWarps][kRsBins];  // per-warp digit counts -> prefix over warps
@@ -207,8 +214,12 @@ size_t radix_sort_workspace_bytes(int64_t n) {
 
 // Sorts (keys, vals) by the low `bits` bits of the keys, stably, ping-ponging with the _alt
 // buffers; returns in *in_alt whether the result ended in the _alt buffers (odd pass count).
+// d_npasses (device, optional): passes [*d_npasses, ceil(bits / 8)) are skipped on the device
+// (their digits are zero in every key: a stable no-op); with an even *d_npasses and an even
+// pass count the result still lands in the input buffers.
 cudaError_t radix_sort_pairs(uint64_t *keys, uint64_t *keys_alt, int32_t *vals, int32_t *vals_alt,
-                             int64_t n, int bits, void *ws, cudaStream_t s, bool *in_alt) {
+                             int64_t n, int bits, void *ws, cudaStream_t s, bool *in_alt,
+                             const int32_t *d_npasses) {
   *in_alt = false;
   if (n <= 0) return cudaSuccess;
   if (n > (int64_t)INT32_MAX) return cudaErrorInvalidValue;
@@ -218,10 +229,12 @@ cudaError_t radix_sort_pairs(uint64_t *keys, uint64_t *keys_alt, int32_t *vals, 
   uint64_t *ka = keys, *kb = keys_alt;
   int32_t *va = vals, *vb = vals_alt;
   for (int shift = 0; shift < bits; shift += kRsBits) {
-    rs_count<<<(unsigned)nt, kRsThreads, 0, s>>>(ka, n, shift, counts, nt);
-    rs_scan_blocks<<<(unsigned)nsb, 1024, 0, s>>>(counts, m, bsum);
-    rs_scan_sums<<<1, 1024, 0, s>>>(bsum, nsb);
-    rs_scatter<<<(unsigned)nt, kRsThreads, 0, s>>>(ka, va, n, shift, counts, bsum, nt, kb, vb);
+    const int pass = shift / kRsBits;
+    rs_count<<<(unsigned)nt, kRsThreads, 0, s>>>(ka, n, shift, counts, nt, d_npasses);
+    rs_scan_blocks<<<(unsigned)nsb, 1024, 0, s>>>(counts, m, bsum, pass, d_npasses);
+    rs_scan_sums<<<1, 1024, 0, s>>>(bsum, nsb, pass, d_npasses);
+    rs_scatter<<<(unsigned)nt, kRsThreads, 0, s>>>(ka, va, n, shift, counts, bsum, nt, kb, vb,
+                                                   d_npasses);
     count_launch(4);
     uint64_t *tk = ka; ka = kb; kb = tk;
     int32_t *tv = va; va = vb; vb = tv;

@@ -565,6 +565,24 @@ def test_capture_shuffled_wide_devices_and_ties():
     assert np.array_equal(got, oracle.capture(a.astype(np.int64), c.astype(np.int64), d))
 
 
+@pytest.mark.parametrize("span_bits,ndev", [(3, 1), (9, 2), (17, 1), (22, 3), (31, 300),
+                                              (38, 7), (45, 1000), (46, 65535)])
+def test_capture_compact_key_widths(span_bits, ndev):
+    # compact sort keys (capture.cu): (device << tb) | (time - tmin) sorted in only
+    # ceil((tb + device bits) / 8) radix passes - odd and even counts from 1 to 8, time
+    # offsets far from zero, equal keys - must give the oracle's records exactly
+    rng = np.random.default_rng(span_bits * 1000 + ndev)
+    n = 20_000
+    t0 = int(rng.integers(0, (1 << 47) - (1 << span_bits) - 16))
+    d = rng.integers(0, ndev, n).astype(np.int32)
+    span = 1 << span_bits
+    a = t0 + rng.integers(0, max(span // 2, 1), n)
+    c = np.minimum(a + 1 + rng.integers(0, max(span // 2, 1), n), t0 + span - 1)
+    c = np.maximum(c, a)
+    got = _gpu_capture(a.astype(np.int64), c.astype(np.int64), d)
+    assert np.array_equal(got, oracle.capture(a.astype(np.int64), c.astype(np.int64), d))
+
+
 def test_capture_full_size_sampled():
     a, c, d = _interleaved_trace(1 << 20, 8, seed=80)
     got = _gpu_capture(a, c, d)
